@@ -1,0 +1,81 @@
+/*
+ * selgen.h -- seeded, counter-based synthetic input generator.
+ *
+ * This module produces INPUT BYTES ONLY: loop-nest descriptors, access
+ * descriptors, launch configurations, device parameter sets and candidates
+ * for the five BASELINE.json configs.  It contains none of the hot path's
+ * arithmetic (no coalescing counts, no Hong & Kim model, no decision).  Both
+ * the CPU oracle (oracle/) and the CUDA path consume its output; neither
+ * includes the other.  The record layouts below are this module's own
+ * definition of the data format; include/sel.h (product) and oracle/oracle.h
+ * (test oracle) declare the same layouts independently and a CPU test checks
+ * that all three agree byte for byte.
+ *
+ * Recipe: DESIGN.md "Input recipe".  Every candidate is a
+ * pure function of (config, candidate index); any rank can generate any
+ * index range without communication.
+ */
+#ifndef SELGEN_H
+#define SELGEN_H
+#include <stdint.h>
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct {                       /* 88 bytes */
+    int32_t num_sms, max_warps_per_sm, max_threads_per_sm, max_blocks_per_sm, regs_per_sm, smem_per_sm;
+    double sm_clock_hz, mem_bw_Bps, link_bw_Bps, launch_overhead_s,
+           mem_ld_cycles, dep_del_coal, dep_del_uncoal, issue_cycles;
+} gen_device_params;
+
+typedef struct {                       /* 64 bytes; all quantities in bytes */
+    int64_t base, c_par[2], c_inner[3];
+    uint8_t elem_bytes, depth, is_store, _pad[13];
+} gen_access;
+
+typedef struct {                       /* 88 bytes */
+    uint64_t P0, P1;
+    uint32_t trip[3];
+    uint8_t par_dims, depth, _pad[2];
+    double comp_insts[4];
+    uint64_t bytes_h2d, bytes_d2h;
+    uint32_t access_off, n_access;
+} gen_nest;
+
+typedef struct {                       /* 16 bytes */
+    uint32_t block, grid_max, regs_per_thread, smem_per_block;
+} gen_launch;
+
+typedef struct {                       /* 24 bytes */
+    uint32_t nest_id;
+    uint16_t launch_id, device_id;
+    double cpu_cycles, cpu_hz;
+} gen_candidate;
+
+/* Config ids follow BASELINE.json "configs" order, 1-based. */
+enum { SELGEN_C1 = 1, SELGEN_C2 = 2, SELGEN_C3 = 3, SELGEN_C4 = 4, SELGEN_C5 = 5 };
+
+/* Number of candidates in the full config (c5: 10^8). */
+uint64_t selgen_num_candidates(int cfg);
+/* The four device parameter sets (K80 one GK210, P100, V100, B200). Returns 4. */
+int selgen_device_sets(gen_device_params* out);
+/* Launch table of a config (c1..c3: 1 entry, c4/c5: 8). Returns the count. */
+int selgen_launches(int cfg, gen_launch* out);
+/* Sizes of the nest/access tables needed for candidates [c0, c1). */
+int selgen_count(int cfg, uint64_t c0, uint64_t c1, uint64_t* n_nests, uint64_t* n_access);
+/* Fill candidates [c0, c1) and the nest/access tables they reference
+ * (nest ids are local to the slice).  Returns 0 or -1 on bad arguments. */
+int selgen_fill(int cfg, uint64_t c0, uint64_t c1,
+                gen_candidate* cands, gen_nest* nests, gen_access* acc);
+/* Shape catalogue (24 Polybench-style sub-kernels). */
+int selgen_num_shapes(void);
+const char* selgen_shape_name(int s);
+/* Counter-based generator: splitmix64(seed ^ (i * golden)). */
+uint64_t selgen_rng(uint64_t seed, uint64_t i);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

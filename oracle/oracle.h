@@ -1,0 +1,92 @@
+/*
+ * oracle.h -- TEST INFRASTRUCTURE ONLY.  Plain, slow CPU oracle for the
+ * batched GPU-side offload-model evaluation (Chikin et al., IPDPSW 2019).
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+ * --impl reference legs may load it.  It shares no code (no header, no
+ * helper, no constant) with the CUDA path in paper_conf_ipps_chikinaat19_b200/;
+ * the record layouts below are declared here independently and checked
+ * against the generator's and the product's by tests/test_layout.py.
+ */
+#ifndef SEL_ORACLE_H
+#define SEL_ORACLE_H
+#include <stdint.h>
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct {
+    int32_t num_sms, max_warps_per_sm, max_threads_per_sm, max_blocks_per_sm, regs_per_sm, smem_per_sm;
+    double sm_clock_hz, mem_bw_Bps, link_bw_Bps, launch_overhead_s,
+           mem_ld_cycles, dep_del_coal, dep_del_uncoal, issue_cycles;
+} or_device;
+
+typedef struct {
+    int64_t base, c_par[2], c_inner[3];
+    uint8_t elem_bytes, depth, is_store, _pad[13];
+} or_access;
+
+typedef struct {
+    uint64_t P0, P1;
+    uint32_t trip[3];
+    uint8_t par_dims, depth, _pad[2];
+    double comp_insts[4];
+    uint64_t bytes_h2d, bytes_d2h;
+    uint32_t access_off, n_access;
+} or_nest;
+
+typedef struct { uint32_t block, grid_max, regs_per_thread, smem_per_block; } or_launch;
+
+typedef struct {
+    uint32_t nest_id;
+    uint16_t launch_id, device_id;
+    double cpu_cycles, cpu_hz;
+} or_candidate;
+
+/* Everything the oracle computes for one candidate: the hot path's outputs
+ * (counts, cycles, t_gpu, decision, status) plus the model's intermediate
+ * values, exposed so that tests can pin them against closed forms. */
+typedef struct {
+    /* a1-a4 counts */
+    uint64_t W, L, S, C, U, WR;
+    /* a1 geometry, a5 occupancy */
+    uint64_t G, T, R, wpb, abps, active_sms, M_it;
+    double N, Rep;
+    /* a4 / a6 intermediates */
+    double comp, mem, MemL_u, MemL_c, MemL, Dep, MWPnb, BWpw, MWPbw, MWP, Comp, Mem, CWP, E;
+    int32_t hk_case;                     /* 0: W == 0 (R22), 1, 2, 3 as in Fig. 4 */
+    /* outputs */
+    double cycles, t_gpu, t_cpu;
+    uint8_t decision, status, _pad[6];
+} or_result;
+
+enum { OR_OK = 0, OR_EINVAL = 1, OR_ERANGE = 2, OR_ELAUNCH = 3 };
+
+/* a1 geometry of a launch (reading R6/R27): out = {G, T, R, wpb}. */
+void oracle_geometry(uint64_t P, uint32_t B, uint32_t grid_max, uint64_t out[4]);
+
+/* Full evaluation of n candidates (brute-force counting + literal model).
+ * threads <= 0 means "all host cores".  Returns 0, or -1 on bad arguments
+ * (null pointers, invalid device parameter set). */
+int oracle_evaluate(const or_device* devs, int n_devs,
+                    const or_candidate* cands, uint64_t n,
+                    const or_nest* nests, uint64_t n_nests,
+                    const or_access* acc, uint64_t n_acc,
+                    const or_launch* launches, uint64_t n_launches,
+                    or_result* out, int threads);
+
+/* The model part only (a4-a7) for given counts r->{W,L,S,C,U,WR}: fills the
+ * rest of *r.  Used by tests to pin the Hong & Kim arithmetic on hand-made
+ * counts. */
+void oracle_model(const or_device* dev, const or_nest* nest, const or_access* acc,
+                  const or_launch* launch, const or_candidate* cand, or_result* r);
+
+/* Layout self-description for tests/test_layout.py. */
+size_t oracle_sizeof(int which);
+size_t oracle_offsetof(int which, int field);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

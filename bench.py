@@ -1,0 +1,329 @@
+#!/usr/bin/env python
+"""Benchmark of the batched GPU-side offload-model evaluation (one JSON line).
+
+Workload (BASELINE.json configs[4], the configuration the metric is quoted
+on): the c5 sweep of 10^8 candidates (24 Polybench-shaped loop nests x
+index-derived trip counts x 8 launch configurations x 4 device parameter
+sets), synthetic and seeded (gen/).  A step is one
+pass of the whole hot path over the batch: per-warp coalescing counts, Hong &
+Kim cycles and the CPU-or-GPU decision for every candidate, plus the NCCL
+all-gather of the decisions when N > 1.  The batch is fixed and sharded
+across ranks by candidate index ("scaling": "strong").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "model evaluations/sec and warp-accesses analysed/sec at 1/2/4/8 B200 (% roofline)"
+UNIT = "evals/s"
+WORKLOAD = ("c5: 10^8-candidate selection sweep (24 Polybench-shaped nests x trip counts x "
+            "8 launch configs x 4 device sets)")
+OPS_PER_WA = 224           # 7 integer lane-ops x 32 lanes per warp-access
+INT_LANES_PER_CLK_SM = 64  # ALU pipe: 4 SMSPs x 16 lanes (rt 2 cyc / warp instr), DESIGN.md "Roofline"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", type=int, default=5)
+    p.add_argument("--candidates", type=int, default=0, help="override the batch size (testing)")
+    p.add_argument("--flags", type=int, default=0, help="libsel flags (1 no count sharing, 2 match_any)")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=15.0)
+    return p.parse_args()
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        sm, smax, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                smax = max(smax, float(f[1]))
+            except ValueError:
+                continue
+            for name, v in zip(names, f[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- helpers
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def ncu_traffic_per_launch():
+    """dram bytes per counting-kernel launch from the committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_count_kernel.json")) as f:
+            return json.load(f).get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+def cpu_oracle_sample(batch, seconds: float, total_candidates: int):
+    """The oracle (as it stands) on a bounded, deterministic sample of the
+    workload, on all host cores."""
+    import oracle
+    cores = os.cpu_count() or 1
+    n = len(batch)
+    cal = max(32, min(256, n))
+    idx = np.linspace(0, n - 1, cal).astype(np.int64)
+    t0 = time.perf_counter()
+    oracle.evaluate(batch.select(idx), threads=cores)
+    t_cal = time.perf_counter() - t0
+    m = int(min(n, max(cal, seconds / max(t_cal / cal, 1e-9))))
+    idx = np.linspace(0, n - 1, m).astype(np.int64)
+    sub = batch.select(idx)
+    t0 = time.perf_counter()
+    r = oracle.evaluate(sub, threads=cores)
+    dt = time.perf_counter() - t0
+    return {"value": m / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{m} candidates evenly spaced over the {total_candidates}-candidate sweep "
+                      f"({int(r['W'].sum())} warp-accesses, {dt:.1f} s)",
+            "wa_per_s": float(r["W"].sum()) / dt}
+
+
+# ---------------------------------------------------------------- reference arm
+def run_reference(args):
+    """--impl reference: the CPU oracle timed as it stands on the same workload,
+    each step a bounded sample (rank 0 only)."""
+    import gen
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    total = gen.num_candidates(args.config) if not args.candidates else args.candidates
+    cores = os.cpu_count() or 1
+    # size a step to ~6 s of host time, calibrated on a strided probe
+    probe_idx = np.linspace(0, total - 1, 96).astype(np.int64)
+    t0 = time.perf_counter()
+    oracle.evaluate(gen.generate_indices(args.config, probe_idx), threads=cores)
+    per_cand = (time.perf_counter() - t0) / len(probe_idx)
+    per_step = int(max(32, min(total, 6.0 / max(per_cand, 1e-9))))
+    stride = max(1, total // per_step)
+    times, evals, was = [], 0, 0
+    for step in range(args.warmup + args.steps):
+        off = (step * 7919) % stride
+        cidx = np.arange(off, total, stride)[:per_step]
+        b = gen.generate_indices(args.config, cidx)
+        t0 = time.perf_counter()
+        r = oracle.evaluate(b, threads=cores)
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+            evals += len(b)
+            was += int(r["W"].sum())
+    T = sum(times)
+    value = evals / T
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64+f64",
+            "data": "synthetic", "config": {"workload": WORKLOAD, "candidates": total},
+            "wa_analysed_per_s": was / T,
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": f"each step {per_step} candidates strided over the {total}-candidate sweep"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def run_ours(args):
+    import torch
+
+    import gen
+    import paper_conf_ipps_chikinaat19_b200 as sel
+    from paper_conf_ipps_chikinaat19_b200 import dist as D
+
+    rank, world, local = D.init()
+    dev = torch.device("cuda", local)
+    total = gen.num_candidates(args.config) if not args.candidates else args.candidates
+    c0, c1 = D.shard_range(total, rank, world)
+    t_gen = time.perf_counter()
+    batch = gen.generate(args.config, c0, c1)
+    t_gen = time.perf_counter() - t_gen
+    ev = sel.Evaluator((batch.nests, batch.accesses, batch.launches, batch.devices), len(batch), args.flags,
+                       device=dev)
+    cands_host = torch.from_numpy(batch.cands.view(np.uint8).reshape(-1)).pin_memory()
+    cands = cands_host.to(dev)
+    stream = torch.cuda.current_stream(dev)
+    out = None
+    gathered = torch.empty(D.padded_len(total, world) * world, dtype=torch.uint8, device=dev) if world > 1 else None
+
+    def step():
+        nonlocal out
+        out = ev.evaluate(cands, out=out)
+        if world > 1:
+            D.gather_decisions(out["decision"], total, world, out=gathered)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+    stats = ev.stats()
+    sel.profile_enable(True)
+    sel.profile_read()
+    launches0 = sel.kernel_launches()
+    D.barrier(world)
+    torch.cuda.synchronize(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+    D.barrier(world)
+    ms_local = e0.elapsed_time(e1)
+    launches = sel.kernel_launches() - launches0
+    count_ms, count_launches = sel.profile_read()
+    sel.profile_enable(False)
+    ms = D.max_over_ranks(ms_local, world, dev)
+    wa_analysed = D.sum_over_ranks(stats["wa_analysed"], world, dev)
+    wa_covered = D.sum_over_ranks(stats["wa_covered"], world, dev)
+    n_invalid = D.sum_over_ranks(stats["n_invalid"], world, dev)
+    t_step = ms / 1e3 / args.steps
+    clocks = clk.summary()
+
+    # ---- end to end through the public API: pinned host inputs -> decisions + cycles on the host
+    e2e = None
+    if not args.no_e2e:
+        nests_h = torch.from_numpy(batch.nests.view(np.uint8).reshape(-1)).pin_memory()
+        acc_h = torch.from_numpy(batch.accesses.view(np.uint8).reshape(-1)).pin_memory()
+        out_host = {"decision": torch.empty(len(batch), dtype=torch.uint8, pin_memory=True),
+                    "cycles": torch.empty(len(batch), dtype=torch.float64, pin_memory=True)}
+        h2d = cands_host.numel() + nests_h.numel() + acc_h.numel()
+        d2h = len(batch) * 9
+
+        def e2e_step():
+            ev.tables.nests.copy_(nests_h, non_blocking=True)
+            ev.tables.accesses.copy_(acc_h, non_blocking=True)
+            ev.evaluate_host(cands_host, out_host=out_host)
+
+        for _ in range(max(1, args.warmup)):
+            e2e_step()
+        torch.cuda.synchronize(dev)
+        D.barrier(world)
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.steps):
+            e2e_step()
+        f1.record(stream)
+        torch.cuda.synchronize(dev)
+        ms_e2e = D.max_over_ranks(f0.elapsed_time(f1), world, dev)
+        e2e = {"value": total / (ms_e2e / 1e3 / args.steps), "unit": UNIT,
+               "h2d_bytes_per_step": D.sum_over_ranks(h2d, world, dev),
+               "d2h_bytes_per_step": D.sum_over_ranks(d2h, world, dev),
+               "ms_per_step": ms_e2e / args.steps}
+
+    if rank != 0:
+        return
+    # ---- roofline of the counting kernel (ALU-pipe bound)
+    f_mhz = clocks["sm_mhz"] or measured_peaks().get("clocks_under_load", {}).get("sm_mhz_median", 1965.0)
+    peak_ops = 148 * INT_LANES_PER_CLK_SM * f_mhz * 1e6
+    wa_per_launch = stats["wa_analysed"]             # this rank's launch (rank 0)
+    avg_count_ms = count_ms / max(count_launches, 1)
+    achieved = wa_per_launch * OPS_PER_WA / (avg_count_ms / 1e3) / 1e12
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak_ops / 1e12, "unit": "Tops/s",
+                "frac": achieved * 1e12 / peak_ops, "traffic": ncu_traffic_per_launch(),
+                "kernel": "sel::k_count<false>", "count_ms_per_launch": avg_count_ms,
+                "count_share_of_step": avg_count_ms / (t_step * 1e3),
+                "peak_source": f"148 SM x {INT_LANES_PER_CLK_SM} INT32 lanes/clk (ALU pipe) x {f_mhz:.0f} MHz "
+                               "median SM clock sampled during the timed region",
+                "algorithmic_ops_per_wa": OPS_PER_WA}
+    hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
+    line = {"metric": METRIC, "value": total / t_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_step * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "candidates": total, "count_sharing": not (args.flags & 1),
+                       "counting_primitive": "match_any" if args.flags & 2 else "residue",
+                       "l2": "inputs larger than L2 (2.4 GB of candidates per pass)",
+                       "parallelism": f"dp{world} (candidate shards) + NCCL all-gather of decisions"},
+            "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
+            "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
+            "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,
+            "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
+    if not args.no_cpu_baseline and world == 1:
+        line["cpu_baseline"] = cpu_oracle_sample(batch, args.cpu_seconds, total)
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+    try:
+        import torch.distributed as dist
+        if dist.is_initialized():
+            dist.destroy_process_group()
+    except Exception:
+        pass
+
+
+if __name__ == "__main__":
+    main()

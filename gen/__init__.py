@@ -75,6 +75,8 @@ def lib():
         L.selgen_fill.argtypes = [ctypes.c_int, u64, u64, vp, vp, vp]
         L.selgen_shape_name.restype = ctypes.c_char_p
         L.selgen_shape_name.argtypes = [ctypes.c_int]
+        L.selgen_count_indices.argtypes = [ctypes.c_int, vp, u64, ctypes.POINTER(u64)]
+        L.selgen_fill_indices.argtypes = [ctypes.c_int, vp, u64, vp, vp, vp]
         L.selgen_rng.restype = u64
         L.selgen_rng.argtypes = [u64, u64]
         _lib = L
@@ -134,6 +136,26 @@ def generate(cfg: int, c0: int = 0, c1: int | None = None) -> Batch:
     acc = np.zeros(max(na.value, 1), ACCESS_DTYPE)
     if L.selgen_fill(cfg, c0, c1, cands.ctypes.data, nests.ctypes.data, acc.ctypes.data) != 0:
         raise ValueError("selgen_fill failed")
+    return Batch(cands, nests, acc, launches(cfg), device_sets())
+
+
+def generate_indices(cfg: int, idx) -> Batch:
+    """Candidates ``idx`` of config 3 or 5 (index-addressable sweeps), each
+    with its own nest copy; for configs 1, 2, 4 the full config is generated
+    and sub-selected."""
+    idx = np.ascontiguousarray(np.asarray(idx, dtype=np.uint64))
+    if cfg not in (3, 5):
+        return generate(cfg).select(idx.astype(np.int64))
+    L = lib()
+    na = ctypes.c_uint64()
+    if L.selgen_count_indices(cfg, idx.ctypes.data, len(idx), ctypes.byref(na)) != 0:
+        raise ValueError("bad candidate index")
+    cands = np.zeros(len(idx), CANDIDATE_DTYPE)
+    nests = np.zeros(max(len(idx), 1), NEST_DTYPE)
+    acc = np.zeros(max(na.value, 1), ACCESS_DTYPE)
+    if L.selgen_fill_indices(cfg, idx.ctypes.data, len(idx), cands.ctypes.data, nests.ctypes.data,
+                             acc.ctypes.data) != 0:
+        raise ValueError("selgen_fill_indices failed")
     return Batch(cands, nests, acc, launches(cfg), device_sets())
 
 

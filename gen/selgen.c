@@ -443,3 +443,32 @@ int selgen_fill(int cfg, uint64_t c0, uint64_t c1, gen_candidate* cands, gen_nes
     }
     return -1;
 }
+
+/* Candidates idx[0..m) of an index-addressable config (c3, c5), each with
+ * its own copy of the nest it references (nests[i], accesses from a running
+ * offset).  Used to draw bounded, strided samples of a sweep. */
+int selgen_count_indices(int cfg, const uint64_t* idx, uint64_t m, uint64_t* n_access) {
+    uint64_t na = 0;
+    for (uint64_t i = 0; i < m; i++) {
+        if (idx[i] >= selgen_num_candidates(cfg)) return -1;
+        if (cfg == SELGEN_C5) na += (uint64_t)SHAPES[(idx[i] / 32) % 24].n_acc;
+        else if (cfg == SELGEN_C3) na += 1;
+        else return -1;
+    }
+    *n_access = na;
+    return 0;
+}
+
+int selgen_fill_indices(int cfg, const uint64_t* idx, uint64_t m, gen_candidate* cands, gen_nest* nests,
+                        gen_access* acc) {
+    uint64_t off = 0;
+    for (uint64_t i = 0; i < m; i++) {
+        uint64_t c = idx[i], na = 0, nn = 0;
+        if (selgen_count(cfg, c, c + 1, &nn, &na) != 0) return -1;
+        if (selgen_fill(cfg, c, c + 1, &cands[i], &nests[i], &acc[off]) != 0) return -1;
+        nests[i].access_off = (uint32_t)off;
+        cands[i].nest_id = (uint32_t)i;
+        off += na;
+    }
+    return 0;
+}

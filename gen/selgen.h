@@ -69,6 +69,11 @@ int selgen_count(int cfg, uint64_t c0, uint64_t c1, uint64_t* n_nests, uint64_t*
  * (nest ids are local to the slice).  Returns 0 or -1 on bad arguments. */
 int selgen_fill(int cfg, uint64_t c0, uint64_t c1,
                 gen_candidate* cands, gen_nest* nests, gen_access* acc);
+/* Arbitrary candidate indices of an index-addressable config (c3, c5); each
+ * candidate gets its own nest copy (nest_id = position in idx). */
+int selgen_count_indices(int cfg, const uint64_t* idx, uint64_t m, uint64_t* n_access);
+int selgen_fill_indices(int cfg, const uint64_t* idx, uint64_t m, gen_candidate* cands, gen_nest* nests,
+                        gen_access* acc);
 /* Shape catalogue (24 Polybench-style sub-kernels). */
 int selgen_num_shapes(void);
 const char* selgen_shape_name(int s);

@@ -1,0 +1,229 @@
+"""B200-native batched GPU-side offload-model evaluation (Chikin et al., IPDPSW 2019).
+
+Thin Python layer over the C ABI of libsel.so (include/sel.h).  Torch is
+used for device memory and streams only; every step of the hot path -- the
+per-warp coalescing counts, the Hong & Kim MWP/CWP cycle prediction with
+#OMP_Rep and the CPU-or-GPU decision -- runs in the sm_100a kernels behind
+the ABI.  There is no CPU fallback: without libsel.so or a GPU these calls
+raise.
+
+Records are passed as raw bytes: numpy structured arrays or torch uint8
+tensors whose layout is the one declared in include/sel.h (the generator in
+gen/ produces exactly that layout).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import (DECISION_CPU, DECISION_GPU, DECISION_INVALID, SEL_EINTERNAL, SEL_EINVAL, SEL_ELAUNCH,
+                   SEL_ERANGE, SEL_F_MATCH_ANY, SEL_F_NO_DEDUP, SEL_OK, SelError)
+
+__all__ = ["load_device_params", "workspace_size", "DeviceTables", "count_transactions", "predict_gpu_cycles",
+           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "kernel_launches",
+           "Evaluator", "SelError", "SEL_F_NO_DEDUP", "SEL_F_MATCH_ANY", "DECISION_CPU", "DECISION_GPU",
+           "DECISION_INVALID", "SEL_OK", "SEL_EINVAL", "SEL_ERANGE", "SEL_ELAUNCH", "SEL_EINTERNAL"]
+
+_REC_SIZE = {"device": 88, "access": 64, "nest": 88, "launch": 16, "candidate": 24, "counts": 48}
+
+
+def _as_bytes_tensor(x, rec: str, device="cuda") -> torch.Tensor:
+    """numpy structured array / bytes tensor -> contiguous uint8 tensor on ``device``."""
+    if isinstance(x, torch.Tensor):
+        t = x.view(torch.uint8) if x.dtype != torch.uint8 else x
+        t = t.reshape(-1)
+    else:
+        a = np.ascontiguousarray(x)
+        if a.dtype.itemsize != _REC_SIZE[rec]:
+            raise ValueError(f"{rec} records must be {_REC_SIZE[rec]} bytes, got {a.dtype.itemsize}")
+        t = torch.from_numpy(a.view(np.uint8).reshape(-1))
+    if t.numel() % _REC_SIZE[rec]:
+        raise ValueError(f"{rec} buffer is not a whole number of records")
+    if device is not None and (t.device.type != torch.device(device).type):
+        t = t.to(device, non_blocking=True)
+    return t.contiguous()
+
+
+def _n(t: torch.Tensor, rec: str) -> int:
+    return t.numel() // _REC_SIZE[rec]
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _require_cuda(*ts):
+    for t in ts:
+        if t is not None and t.device.type != "cuda":
+            raise ValueError("libsel arguments must be CUDA tensors")
+
+
+# ------------------------------------------------------------------ API
+def load_device_params(sets) -> None:
+    """sel_load_device_params: copy 1..16 device parameter sets (host)."""
+    a = np.ascontiguousarray(sets)
+    if a.dtype.itemsize != _REC_SIZE["device"]:
+        raise ValueError("device parameter records must be 88 bytes")
+    _lib.check(_lib.lib().sel_load_device_params(a.ctypes.data, len(a)))
+
+
+def workspace_size(n: int, n_nests: int, flags: int = 0) -> int:
+    return int(_lib.lib().sel_workspace_size(n, n_nests, flags))
+
+
+def alloc_workspace(n: int, n_nests: int, flags: int = 0, device="cuda") -> torch.Tensor:
+    nbytes = workspace_size(n, n_nests, flags)
+    return torch.empty(nbytes + 256, dtype=torch.uint8, device=device)
+
+
+def _ws_ptr(ws: torch.Tensor):
+    p = ws.data_ptr()
+    return ctypes.c_void_p((p + 255) & ~255), ws.numel() - (((p + 255) & ~255) - p)
+
+
+class DeviceTables:
+    """Device copies of the shared descriptor tables (nests, accesses, launches)."""
+
+    def __init__(self, nests, accesses, launches, device="cuda"):
+        self.nests = _as_bytes_tensor(nests, "nest", device)
+        self.accesses = _as_bytes_tensor(accesses, "access", device)
+        self.launches = _as_bytes_tensor(launches, "launch", device)
+        self.n_nests = _n(self.nests, "nest")
+        self.c = _lib.Tables(self.nests.data_ptr(), self.n_nests, self.accesses.data_ptr(),
+                             _n(self.accesses, "access"), self.launches.data_ptr(), _n(self.launches, "launch"))
+
+    def ref(self):
+        return ctypes.byref(self.c)
+
+
+def count_transactions(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor, flags: int = 0,
+                       out=None, status=None, stream=None):
+    """sel_count_transactions -> (counts int64[n, 6], status uint8[n])."""
+    _require_cuda(cands, workspace)
+    n = _n(cands, "candidate")
+    dev = cands.device
+    out = torch.empty((n, 6), dtype=torch.int64, device=dev) if out is None else out
+    status = torch.empty(n, dtype=torch.uint8, device=dev) if status is None else status
+    wp, wb = _ws_ptr(workspace)
+    _lib.check(_lib.lib().sel_count_transactions(_ptr(cands), n, tables.ref(), _ptr(out), _ptr(status), wp, wb,
+                                                 flags, _stream(stream)))
+    return out, status
+
+
+def predict_gpu_cycles(cands: torch.Tensor, tables: DeviceTables, counts: torch.Tensor, status: torch.Tensor,
+                       want_t_gpu: bool = True, stream=None):
+    """sel_predict_gpu_cycles -> (cycles f64[n], t_gpu f64[n] | None); status is updated in place."""
+    _require_cuda(cands, counts, status)
+    n = _n(cands, "candidate")
+    cycles = torch.empty(n, dtype=torch.float64, device=cands.device)
+    t_gpu = torch.empty(n, dtype=torch.float64, device=cands.device) if want_t_gpu else None
+    _lib.check(_lib.lib().sel_predict_gpu_cycles(_ptr(cands), n, tables.ref(), _ptr(counts), _ptr(cycles),
+                                                 _ptr(t_gpu), _ptr(status), _stream(stream)))
+    return cycles, t_gpu
+
+
+def select(cands: torch.Tensor, t_gpu: torch.Tensor, status: torch.Tensor, stream=None) -> torch.Tensor:
+    """sel_select -> decision uint8[n] (1 GPU, 0 CPU, 0xFF invalid)."""
+    _require_cuda(cands, t_gpu, status)
+    n = _n(cands, "candidate")
+    decision = torch.empty(n, dtype=torch.uint8, device=cands.device)
+    _lib.check(_lib.lib().sel_select(_ptr(cands), n, _ptr(t_gpu), _ptr(status), _ptr(decision), _stream(stream)))
+    return decision
+
+
+def evaluate(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor, flags: int = 0,
+             want_counts: bool = False, want_t_gpu: bool = False, out: dict | None = None, stream=None) -> dict:
+    """sel_evaluate (fused a1-a7) -> dict of decision, cycles, status [, t_gpu, counts]."""
+    _require_cuda(cands, workspace)
+    n = _n(cands, "candidate")
+    dev = cands.device
+    if out is None:
+        out = {"decision": torch.empty(n, dtype=torch.uint8, device=dev),
+               "cycles": torch.empty(n, dtype=torch.float64, device=dev),
+               "status": torch.empty(n, dtype=torch.uint8, device=dev)}
+        if want_t_gpu:
+            out["t_gpu"] = torch.empty(n, dtype=torch.float64, device=dev)
+        if want_counts:
+            out["counts"] = torch.empty((n, 6), dtype=torch.int64, device=dev)
+    wp, wb = _ws_ptr(workspace)
+    _lib.check(_lib.lib().sel_evaluate(_ptr(cands), n, tables.ref(), _ptr(out["decision"]), _ptr(out["cycles"]),
+                                       _ptr(out.get("t_gpu")), _ptr(out.get("counts")), _ptr(out["status"]), wp, wb,
+                                       flags, _stream(stream)))
+    return out
+
+
+def read_stats(workspace: torch.Tensor, stream=None) -> dict:
+    st = _lib.Stats()
+    wp, _ = _ws_ptr(workspace)
+    _lib.check(_lib.lib().sel_read_stats(wp, ctypes.byref(st), _stream(stream)))
+    return {k: int(getattr(st, k)) for k in ("n_candidates", "n_problems", "wa_analysed", "wa_covered",
+                                             "n_invalid")}
+
+
+def profile_enable(on: bool = True) -> None:
+    _lib.check(_lib.lib().sel_profile_enable(1 if on else 0))
+
+
+def profile_read():
+    """-> (counting-kernel milliseconds, counting launches) since the last read."""
+    ms, k = ctypes.c_double(), ctypes.c_uint64()
+    _lib.check(_lib.lib().sel_profile_read(ctypes.byref(ms), ctypes.byref(k)))
+    return ms.value, k.value
+
+
+def kernel_launches() -> int:
+    return int(_lib.lib().sel_kernel_launches())
+
+
+# same names as the C ABI
+sel_load_device_params = load_device_params
+sel_workspace_size = workspace_size
+sel_count_transactions = count_transactions
+sel_predict_gpu_cycles = predict_gpu_cycles
+sel_select = select
+sel_evaluate = evaluate
+sel_read_stats = read_stats
+
+
+class Evaluator:
+    """Convenience holder: device tables + a workspace sized for up to
+    ``max_n`` candidates.  ``evaluate`` takes device candidates;
+    ``evaluate_host`` takes host (ideally pinned) candidates and copies them
+    in and the decisions/cycles out on the same stream (end-to-end path)."""
+
+    def __init__(self, batch_tables, max_n: int, flags: int = 0, device="cuda"):
+        nests, accesses, launches, devices = batch_tables
+        load_device_params(devices)
+        self.tables = DeviceTables(nests, accesses, launches, device)
+        self.flags = flags
+        self.max_n = max_n
+        self.workspace = alloc_workspace(max_n, self.tables.n_nests, flags, device)
+        self.device = device
+
+    def evaluate(self, cands: torch.Tensor, **kw) -> dict:
+        if _n(cands, "candidate") > self.max_n:
+            raise ValueError("batch larger than the workspace")
+        return evaluate(cands, self.tables, self.workspace, self.flags, **kw)
+
+    def evaluate_host(self, cands_host: torch.Tensor, out_host: dict | None = None, stream=None) -> dict:
+        """H2D copy of the candidates, sel_evaluate, D2H copy of decision and cycles."""
+        n = _n(cands_host, "candidate")
+        d = cands_host.to(self.device, non_blocking=True)
+        res = self.evaluate(d)
+        if out_host is None:
+            out_host = {"decision": torch.empty(n, dtype=torch.uint8, pin_memory=True),
+                        "cycles": torch.empty(n, dtype=torch.float64, pin_memory=True)}
+        out_host["decision"].copy_(res["decision"], non_blocking=True)
+        out_host["cycles"].copy_(res["cycles"], non_blocking=True)
+        return out_host
+
+    def stats(self) -> dict:
+        return read_stats(self.workspace)

@@ -1,0 +1,147 @@
+// sel_device.cuh -- device-side helpers shared by the libsel kernels:
+// validation rules V1-V7, launch geometry (a1,
+// P:L225; readings R6-R9, R27) and the workspace layout.  No host code.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "../../include/sel.h"
+
+namespace sel {
+
+constexpr uint32_t kFull = 0xffffffffu;
+constexpr uint64_t kLim62 = 1ull << 62;
+constexpr uint64_t kLim48 = 1ull << 48;
+constexpr uint64_t kLim40 = 1ull << 40;
+constexpr uint32_t kNoProblem = 0xffffffffu;
+constexpr int kSlots = 8;              // distinct B classes shared per nest before overflow
+
+// ------------------------------------------------------------------ workspace
+// All offsets are 256-byte aligned.  Sized for the worst case of one counting
+// problem per candidate.
+struct WsHeader {
+    sel_stats stats;                   // 64 B, read by sel_read_stats
+    unsigned long long n_problems;     // device-side problem count
+    unsigned long long chunk_ctr;      // dynamic work counter of the count kernel
+    unsigned int n_overflow;           // problems allocated past the slot table
+    unsigned int _pad0;
+    unsigned long long _pad[21];
+};
+static_assert(sizeof(WsHeader) == 256, "header size");
+
+struct WsLayout {
+    size_t hdr, slots, nest_base, cand_pid, prob_nest, prob_B, prob_W, prob_WR, prob_cnt,
+        prob_status, cand_status, scan_tmp, total;
+};
+
+__host__ __device__ inline size_t ws_align(size_t x) { return (x + 255) & ~size_t(255); }
+
+// Number of scan partial sums for n items (kScanItems per block).
+constexpr int kScanThreads = 256;
+constexpr int kScanPer = 8;
+constexpr uint64_t kScanItems = uint64_t(kScanThreads) * kScanPer;
+__host__ __device__ inline uint64_t scan_blocks(uint64_t n) { return (n + kScanItems) / kScanItems + 1; }
+
+__host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint32_t flags) {
+    WsLayout L{};
+    bool dedup = !(flags & SEL_F_NO_DEDUP);
+    size_t o = 0;
+    L.hdr = o;        o = ws_align(o + sizeof(WsHeader));
+    L.slots = o;      o = ws_align(o + (dedup ? n_nests * kSlots * sizeof(uint32_t) : 0));
+    L.nest_base = o;  o = ws_align(o + (dedup ? (n_nests + 1) * sizeof(uint64_t) : 0));
+    L.cand_pid = o;   o = ws_align(o + n * sizeof(uint32_t));
+    L.prob_nest = o;  o = ws_align(o + n * sizeof(uint32_t));
+    L.prob_B = o;     o = ws_align(o + n * sizeof(uint32_t));
+    L.prob_W = o;     o = ws_align(o + (n + 1) * sizeof(uint64_t));
+    L.prob_WR = o;    o = ws_align(o + n * sizeof(uint64_t));
+    L.prob_cnt = o;   o = ws_align(o + n * 5 * sizeof(uint64_t));
+    L.prob_status = o; o = ws_align(o + n);
+    L.cand_status = o; o = ws_align(o + n);
+    uint64_t big = n > n_nests ? n : n_nests;
+    L.scan_tmp = o;   o = ws_align(o + scan_blocks(big) * sizeof(uint64_t) * 2);
+    L.total = o;
+    return L;
+}
+
+// ------------------------------------------------------------------- basics
+__device__ __forceinline__ uint64_t eff_trip(uint32_t t) {
+    return t == SEL_TRIP_UNKNOWN ? 128ull : uint64_t(t);
+}
+__device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return a / b + (a % b != 0); }
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint64_t smul(uint64_t a, uint64_t b) {
+    if (a == 0 || b == 0) return 0;
+    return (a > ~0ull / b) ? ~0ull : a * b;
+}
+__device__ __forceinline__ uint64_t sadd(uint64_t a, uint64_t b) { return (a > ~0ull - b) ? ~0ull : a + b; }
+__device__ __forceinline__ uint64_t uabs(int64_t v) { return v < 0 ? 0ull - uint64_t(v) : uint64_t(v); }
+
+// B class for count sharing: counts depend on B only when 32 does not divide
+// it (every warp is then an aligned 32-iteration chunk of p-space), and never
+// on G_max or the device.
+__device__ __forceinline__ uint32_t b_class(uint32_t B) { return (B & 31u) == 0 ? 32u : B; }
+
+// Candidate-level checks V1, V2 (ids, host clock, launch bounds).
+__device__ __forceinline__ uint8_t validate_candidate(const sel_candidate& c, const sel_tables& t,
+                                                      int n_sets) {
+    if (c.nest_id >= t.n_nests || c.launch_id >= t.n_launches || c.device_id >= uint32_t(n_sets) ||
+        !(c.cpu_hz > 0.0))
+        return SEL_EINVAL;
+    const sel_launch l = t.launches[c.launch_id];
+    if (l.block < 1 || l.block > 1024 || l.grid_max < 1) return SEL_EINVAL;
+    return SEL_OK;
+}
+
+// Nest-level checks V3-V6; on success *M_it = sum_k prod_{j<depth_k} T_j.
+__device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc_all, uint64_t n_acc_total,
+                                        uint64_t* M_it_out) {
+    if ((n.par_dims != 1 && n.par_dims != 2) || n.depth > 3 || (n.par_dims == 1 && n.P1 != 1) ||
+        uint64_t(n.access_off) + uint64_t(n.n_access) > n_acc_total)
+        return SEL_EINVAL;
+    const uint64_t P = smul(n.P0, n.P1);
+    if (n.P0 >= kLim40 || P >= kLim40) return SEL_ERANGE;
+    uint64_t T[3];
+    for (int j = 0; j < 3; j++) T[j] = eff_trip(n.trip[j]);
+    const sel_access* acc = acc_all + n.access_off;
+    for (uint32_t k = 0; k < n.n_access; k++) {
+        const sel_access a = acc[k];
+        const int64_t e = a.elem_bytes;
+        if (!(e == 1 || e == 2 || e == 4 || e == 8 || e == 16) || a.depth > n.depth) return SEL_EINVAL;
+        // power-of-two element size: divisibility by masking
+        const int64_t m = e - 1;
+        bool bad = (a.base & m) || (a.c_par[0] & m) || (n.par_dims == 2 && (a.c_par[1] & m));
+        for (int j = 0; j < a.depth; j++) bad |= (a.c_inner[j] & m) != 0;
+        if (bad) return SEL_EINVAL;
+    }
+    uint64_t M_it = 0;
+    for (uint32_t k = 0; k < n.n_access; k++) {
+        const sel_access a = acc[k];
+        const uint64_t e0 = (n.par_dims == 1) ? P : n.P0;
+        uint64_t bound = uabs(a.base);
+        bound = sadd(bound, smul(uabs(a.c_par[0]), e0 ? e0 - 1 : 0));
+        if (n.par_dims == 2) bound = sadd(bound, smul(uabs(a.c_par[1]), n.P1 ? n.P1 - 1 : 0));
+        uint64_t Mk = 1;
+        for (int j = 0; j < a.depth; j++) {
+            bound = sadd(bound, smul(uabs(a.c_inner[j]), T[j] ? T[j] - 1 : 0));
+            Mk = smul(Mk, T[j]);
+        }
+        if (bound >= kLim62) return SEL_ERANGE;
+        M_it = sadd(M_it, Mk);
+    }
+    if (smul(P, M_it) >= kLim48) return SEL_ERANGE;
+    *M_it_out = M_it;
+    return SEL_OK;
+}
+
+// Warps with at least one active lane (R8, R9), summed over the R*G blocks of
+// the launch.  Block k covers iterations [kB, kB + B); block-to-grid mapping
+// (R7) does not change which iterations share a warp, so WR depends only on
+// P and B.
+__device__ __forceinline__ uint64_t warp_reps(uint64_t P, uint32_t B) {
+    if (P == 0) return 0;
+    if ((B & 31u) == 0) return cdiv(P, 32);
+    const uint64_t wpb = cdiv(B, 32);
+    const uint64_t nb = cdiv(P, B);
+    return (nb - 1) * wpb + cdiv(P - (nb - 1) * B, 32);
+}
+
+}  // namespace sel

@@ -1,0 +1,276 @@
+// sel_plan.cu -- turns a batch of candidates into counting problems.
+//
+// Counts (a1-a3) of a candidate depend only on its nest and on B when
+// 32 does not divide B (every warp is then an aligned 32-iteration chunk of
+// the parallel iteration space), never on G_max or the device set
+// (DESIGN.md "Count sharing").  Candidates that share (nest, B class) are
+// therefore counted once: a per-nest slot table collects the distinct B
+// classes (warp-aggregated with __match_any_sync), the classes are sorted
+// so problem ids are deterministic, and a device-wide scan assigns ids.
+// Each problem then gets its closed-form number of warp-accesses
+// W = WR * M_it, and a second scan turns those into the prefix the counting
+// kernel partitions.  Everything stays on the device (no host sync).
+#include "sel_device.cuh"
+#include "sel_internal.h"
+
+namespace sel {
+
+// ------------------------------------------------------------------- scan
+// Exclusive scan of unsigned 64-bit values in place: x[0..n) -> prefix,
+// x[n] = total.  n is read from *n_dev when given (device-side count).
+__global__ void __launch_bounds__(kScanThreads) k_scan_reduce(const unsigned long long* x, uint64_t n_host,
+                                                              const unsigned long long* n_dev,
+                                                              unsigned long long* partial) {
+    const uint64_t n = n_dev ? *n_dev : n_host;
+    const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
+    unsigned long long s = 0;
+    if (begin < n) {
+        for (int i = 0; i < kScanPer; i++) {
+            uint64_t idx = begin + uint64_t(i) * kScanThreads + threadIdx.x;
+            if (idx < n) s += x[idx];
+        }
+    }
+    __shared__ unsigned long long red[kScanThreads / 32];
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int w = 0; w < kScanThreads / 32; w++) t += red[w];
+        partial[blockIdx.x] = t;
+    }
+}
+
+// single block: exclusive scan of the per-block partial sums
+__global__ void __launch_bounds__(1024) k_scan_partials(unsigned long long* partial, uint64_t nb_host,
+                                                        uint64_t n_host, const unsigned long long* n_dev) {
+    const uint64_t n = n_dev ? *n_dev : n_host;
+    uint64_t nb = (n + kScanItems - 1) / kScanItems;
+    if (nb > nb_host) nb = nb_host;
+    __shared__ unsigned long long wsum[32];
+    __shared__ unsigned long long carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (uint64_t base = 0; base < nb; base += 1024) {
+        uint64_t i = base + threadIdx.x;
+        unsigned long long v = i < nb ? partial[i] : 0, inc = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned long long y = __shfl_up_sync(kFull, inc, o);
+            if ((threadIdx.x & 31) >= o) inc += y;
+        }
+        if ((threadIdx.x & 31) == 31) wsum[threadIdx.x >> 5] = inc;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            unsigned long long w = wsum[threadIdx.x], wi = w;
+            for (int o = 1; o < 32; o <<= 1) {
+                unsigned long long y = __shfl_up_sync(kFull, wi, o);
+                if (threadIdx.x >= o) wi += y;
+            }
+            wsum[threadIdx.x] = wi - w;
+        }
+        __syncthreads();
+        unsigned long long excl = carry + wsum[threadIdx.x >> 5] + inc - v;
+        if (i < nb) partial[i] = excl;
+        __syncthreads();
+        if (threadIdx.x == 1023) carry = excl + v;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) partial[nb] = carry;
+}
+
+__global__ void __launch_bounds__(kScanThreads) k_scan_down(unsigned long long* x, uint64_t n_host,
+                                                            const unsigned long long* n_dev,
+                                                            const unsigned long long* partial) {
+    const uint64_t n = n_dev ? *n_dev : n_host;
+    const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
+    if (begin > n) return;
+    if (begin == n) {                       // the block that owns x[n] = total
+        if (threadIdx.x == 0) x[n] = partial[blockIdx.x];
+        return;
+    }
+    // each thread scans kScanPer consecutive items
+    const uint64_t my = begin + uint64_t(threadIdx.x) * kScanPer;
+    unsigned long long v[kScanPer], s = 0;
+    for (int i = 0; i < kScanPer; i++) {
+        v[i] = (my + i < n) ? x[my + i] : 0;
+        s += v[i];
+    }
+    __shared__ unsigned long long wsum[kScanThreads / 32];
+    unsigned long long inc = s;
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned long long y = __shfl_up_sync(kFull, inc, o);
+        if ((threadIdx.x & 31) >= o) inc += y;
+    }
+    if ((threadIdx.x & 31) == 31) wsum[threadIdx.x >> 5] = inc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long c = 0;
+        for (int w = 0; w < kScanThreads / 32; w++) { unsigned long long t = wsum[w]; wsum[w] = c; c += t; }
+    }
+    __syncthreads();
+    unsigned long long run = partial[blockIdx.x] + wsum[threadIdx.x >> 5] + inc - s;
+    for (int i = 0; i < kScanPer; i++) {
+        if (my + i < n) x[my + i] = run;
+        run += v[i];
+    }
+    const uint64_t last = begin + kScanItems;
+    if (last >= n && threadIdx.x == 0 && n < last) x[n] = partial[blockIdx.x + 1];
+}
+
+static cudaError_t scan_u64(unsigned long long* x, uint64_t n_max, const unsigned long long* n_dev,
+                            unsigned long long* partial, cudaStream_t s) {
+    const uint64_t nb = (n_max + kScanItems) / kScanItems;     // covers index n_max as well
+    k_scan_reduce<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial);
+    k_scan_partials<<<1, 1024, 0, s>>>(partial, nb, n_max, n_dev);
+    k_scan_down<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial);
+    note_launch(3);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ plan
+// V1-V2 per candidate; dedup: insert the candidate's B class into its nest's
+// slot table (one CAS per distinct key per warp).
+__global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict__ cands, uint64_t n,
+                                                sel_tables t, int n_sets, uint32_t* slots,
+                                                uint8_t* cand_status, int dedup, uint32_t* prob_nest,
+                                                uint32_t* prob_B, uint32_t* cand_pid) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t base = uint64_t(blockIdx.x) * blockDim.x; base < n; base += stride) {
+        const uint64_t c = base + threadIdx.x;
+        const bool in = c < n;
+        const unsigned inmask = __ballot_sync(kFull, in);
+        if (!in) continue;
+        const sel_candidate cd = cands[c];
+        const uint8_t st = validate_candidate(cd, t, n_sets);
+        cand_status[c] = st;
+        if (!dedup) {
+            cand_pid[c] = uint32_t(c);
+            prob_nest[c] = st ? kNoProblem : cd.nest_id;
+            prob_B[c] = st ? 0u : t.launches[cd.launch_id].block;
+            continue;
+        }
+        const uint32_t bc = st ? 0u : b_class(t.launches[cd.launch_id].block);
+        const unsigned long long key = st ? ~0ull : ((unsigned long long)cd.nest_id << 32) | bc;
+        const unsigned peers = __match_any_sync(inmask, key);
+        const int leader = __ffs(peers) - 1;
+        if (st == 0 && (threadIdx.x & 31) == leader) {
+            uint32_t* s = slots + uint64_t(cd.nest_id) * kSlots;
+            for (int j = 0; j < kSlots; j++) {
+                uint32_t old = atomicCAS(s + j, 0u, bc);
+                if (old == 0u || old == bc) break;
+            }
+        }
+    }
+}
+
+// sort each nest's B classes (deterministic ids) and count them
+__global__ void __launch_bounds__(256) k_rank_slots(uint32_t* slots, uint64_t n_nests,
+                                                    unsigned long long* nest_cnt) {
+    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (i >= n_nests) return;
+    uint32_t v[kSlots];
+    int m = 0;
+    for (int j = 0; j < kSlots; j++) {
+        uint32_t x = slots[i * kSlots + j];
+        if (x) v[m++] = x;
+    }
+    for (int a = 1; a < m; a++) {
+        uint32_t x = v[a];
+        int b = a - 1;
+        while (b >= 0 && v[b] > x) { v[b + 1] = v[b]; b--; }
+        v[b + 1] = x;
+    }
+    for (int j = 0; j < kSlots; j++) slots[i * kSlots + j] = j < m ? v[j] : 0u;
+    nest_cnt[i] = (unsigned long long)m;
+}
+
+__global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict__ cands, uint64_t n,
+                                                sel_tables t, const uint32_t* slots,
+                                                const unsigned long long* nest_base, uint64_t n_nests,
+                                                const uint8_t* cand_status, uint32_t* cand_pid,
+                                                uint32_t* prob_nest, uint32_t* prob_B, WsHeader* hdr) {
+    const uint64_t c = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (c >= n) return;
+    if (cand_status[c]) { cand_pid[c] = kNoProblem; return; }
+    const sel_candidate cd = cands[c];
+    const uint32_t bc = b_class(t.launches[cd.launch_id].block);
+    const uint32_t* s = slots + uint64_t(cd.nest_id) * kSlots;
+    uint64_t pid = ~0ull;
+    for (int j = 0; j < kSlots; j++) {
+        if (s[j] == bc) { pid = nest_base[cd.nest_id] + j; break; }
+    }
+    if (pid == ~0ull) pid = nest_base[n_nests] + atomicAdd(&hdr->n_overflow, 1u);   // slot table full
+    cand_pid[c] = uint32_t(pid);
+    prob_nest[pid] = cd.nest_id;      // identical values from every sharer
+    prob_B[pid] = bc;
+}
+
+__global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_base, uint64_t n_nests,
+                                uint64_t n, int dedup) {
+    unsigned long long np = dedup ? nest_base[n_nests] + hdr->n_overflow : n;
+    hdr->n_problems = np;
+    hdr->chunk_ctr = 0;
+    hdr->stats.n_candidates = n;
+    hdr->stats.n_problems = np;
+}
+
+// closed-form W = WR * M_it per problem (+ nest validation V3-V6)
+__global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader* hdr, const uint32_t* prob_nest,
+                                                   const uint32_t* prob_B, unsigned long long* prob_W,
+                                                   unsigned long long* prob_WR, uint8_t* prob_status,
+                                                   unsigned long long* prob_cnt) {
+    const uint64_t nq = hdr->n_problems;
+    const uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (q >= nq) return;
+    for (int f = 0; f < 5; f++) prob_cnt[q * 5 + f] = 0;
+    const uint32_t nid = prob_nest[q];
+    if (nid == kNoProblem) { prob_W[q] = 0; prob_WR[q] = 0; prob_status[q] = SEL_EINVAL; return; }
+    const sel_nest nest = t.nests[nid];
+    uint64_t M_it = 0;
+    const uint8_t st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
+    prob_status[q] = st;
+    if (st) { prob_W[q] = 0; prob_WR[q] = 0; return; }
+    const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
+    prob_WR[q] = WR;
+    prob_W[q] = WR * M_it;
+}
+
+__global__ void k_plan_stats(WsHeader* hdr, const unsigned long long* prefix) {
+    hdr->stats.wa_analysed = prefix[hdr->n_problems];
+}
+
+cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables& t, int n_sets,
+                        const WsPtrs& w, uint64_t n_nests, uint32_t flags, cudaStream_t s) {
+    const bool dedup = !(flags & SEL_F_NO_DEDUP);
+    cudaError_t e = cudaMemsetAsync(w.hdr, 0, sizeof(WsHeader), s);
+    if (e != cudaSuccess) return e;
+    if (dedup && n_nests) {
+        e = cudaMemsetAsync(w.slots, 0, n_nests * kSlots * sizeof(uint32_t), s);
+        if (e != cudaSuccess) return e;
+    }
+    const unsigned gb = unsigned((n + 255) / 256 < 148u * 64 ? (n + 255) / 256 : 148u * 64);
+    k_insert<<<gb, 256, 0, s>>>(cands, n, t, n_sets, w.slots, w.cand_status, dedup ? 1 : 0, w.prob_nest,
+                                w.prob_B, w.cand_pid);
+    note_launch();
+    if (dedup) {
+        if (n_nests) {
+            k_rank_slots<<<unsigned((n_nests + 255) / 256), 256, 0, s>>>(w.slots, n_nests, w.nest_base);
+            note_launch();
+        }
+        if ((e = scan_u64(w.nest_base, n_nests, nullptr, w.scan_tmp, s)) != cudaSuccess) return e;
+        k_assign<<<unsigned((n + 255) / 256), 256, 0, s>>>(cands, n, t, w.slots, w.nest_base, n_nests,
+                                                           w.cand_status, w.cand_pid, w.prob_nest, w.prob_B,
+                                                           w.hdr);
+        note_launch();
+    }
+    k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0);
+    k_problem_w<<<unsigned((n + 255) / 256), 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
+                                                          w.prob_status, w.prob_cnt);
+    note_launch(2);
+    if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s)) != cudaSuccess) return e;
+    k_plan_stats<<<1, 1, 0, s>>>(w.hdr, w.prob_W);
+    note_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace sel

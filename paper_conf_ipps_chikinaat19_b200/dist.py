@@ -1,0 +1,90 @@
+"""Multi-GPU plumbing: one process per GPU, candidates sharded by index range.
+
+Candidates are independent: each rank evaluates a contiguous
+range of the candidate index space with no data-path exchange; the only
+collective is the all-gather of the per-candidate decisions the north star
+asks for (NCCL over NVLink / NVSwitch on a GPU box, gloo in the CPU tests).
+Ranges are padded to a common length so a single ``all_gather_into_tensor``
+suffices; padding bytes are dropped after the gather.
+"""
+from __future__ import annotations
+
+import os
+
+import torch
+import torch.distributed as dist
+
+
+def env_rank_world():
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), \
+        int(os.environ.get("LOCAL_RANK", "0"))
+
+
+def init(backend: str | None = None):
+    """Initialise the default process group from the torchrun environment
+    (no-op for a single process).  Returns (rank, world, local_rank)."""
+    rank, world, local = env_rank_world()
+    if world > 1 and not dist.is_initialized():
+        if backend is None:
+            backend = "nccl" if torch.cuda.is_available() else "gloo"
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+            dist.init_process_group(backend, device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(local)
+    return rank, world, local
+
+
+def shard_range(total: int, rank: int, world: int):
+    """Contiguous candidate range [c0, c1) of ``rank``; sizes differ by <= 1.
+    The c5 index interleave (device, launch, kernel in the low digits) makes
+    equal-count ranges near-equal work."""
+    base, rem = divmod(total, world)
+    c0 = rank * base + min(rank, rem)
+    return c0, c0 + base + (1 if rank < rem else 0)
+
+
+def padded_len(total: int, world: int) -> int:
+    return -(-total // world)
+
+
+def gather_decisions(local: torch.Tensor, total: int, world: int, out: torch.Tensor | None = None,
+                     group=None) -> torch.Tensor:
+    """All-gather uint8 decisions of every rank's shard into a ``total``-long
+    vector in candidate order (identical on every rank)."""
+    if world == 1:
+        return local
+    n_pad = padded_len(total, world)
+    buf = torch.zeros(n_pad, dtype=torch.uint8, device=local.device)
+    buf[: local.numel()].copy_(local)
+    full = torch.empty(n_pad * world, dtype=torch.uint8, device=local.device) if out is None else out
+    dist.all_gather_into_tensor(full, buf, group=group)
+    parts = []
+    for r in range(world):
+        c0, c1 = shard_range(total, r, world)
+        parts.append(full[r * n_pad: r * n_pad + (c1 - c0)])
+    return torch.cat(parts)
+
+
+def max_over_ranks(x: float, world: int, device) -> float:
+    if world == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def sum_over_ranks(x: int, world: int, device) -> int:
+    if world == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.int64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return int(t.item())
+
+
+def barrier(world: int):
+    if world > 1:
+        dist.barrier()

@@ -1,0 +1,257 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Bit-exact counts, statuses and decisions; fp64 cycles
+within 1e-6 relative (BASELINE.json north_star) -- in practice bit-exact,
+which is also asserted for the fused path (R30)."""
+import random
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+FIELDS = ["W", "L", "S", "C", "U", "WR"]
+REL_TOL = 1e-6
+
+
+@pytest.fixture(scope="module")
+def sel():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_chikinaat19_b200 as s
+    assert torch.cuda.is_available()
+    return s
+
+
+def run_gpu(sel, b, flags=0, api="fused"):
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), max(len(b), 1), flags)
+    cands = sel._as_bytes_tensor(b.cands, "candidate")
+    if api == "fused":
+        r = ev.evaluate(cands, want_counts=True, want_t_gpu=True)
+    else:
+        counts, status = sel.count_transactions(cands, ev.tables, ev.workspace, flags)
+        cycles, t_gpu = sel.predict_gpu_cycles(cands, ev.tables, counts, status)
+        decision = sel.select(cands, t_gpu, status)
+        r = dict(counts=counts, status=status, cycles=cycles, t_gpu=t_gpu, decision=decision)
+    torch.cuda.synchronize()
+    out = {k: v.cpu().numpy() for k, v in r.items()}
+    out["counts"] = out["counts"].astype(np.uint64)
+    out["stats"] = sel.read_stats(ev.workspace) if api == "fused" else None
+    return out
+
+
+def assert_parity(g, ref, exact_cycles=True, ctx=""):
+    for j, f in enumerate(FIELDS):
+        bad = np.nonzero(g["counts"][:, j] != ref[f])[0]
+        assert len(bad) == 0, f"{ctx}: count {f} differs at {bad[:10]}: gpu {g['counts'][bad[:5], j]} oracle {ref[f][bad[:5]]}"
+    bad = np.nonzero(g["status"] != ref["status"])[0]
+    assert len(bad) == 0, f"{ctx}: status differs at {bad[:10]}: {g['status'][bad[:5]]} vs {ref['status'][bad[:5]]}"
+    bad = np.nonzero(g["decision"] != ref["decision"])[0]
+    assert len(bad) == 0, f"{ctx}: decision differs at {bad[:10]}"
+    rel = np.abs(g["cycles"] - ref["cycles"]) / np.maximum(np.abs(ref["cycles"]), 1e-300)
+    assert (rel <= REL_TOL).all(), f"{ctx}: cycles rel err {rel.max()}"
+    if exact_cycles:
+        assert (g["cycles"] == ref["cycles"]).all(), f"{ctx}: cycles not bit-exact (max rel {rel.max()})"
+        same = (g["t_gpu"] == ref["t_gpu"]) | (np.isinf(g["t_gpu"]) & np.isinf(ref["t_gpu"]))
+        assert same.all(), f"{ctx}: t_gpu not bit-exact"
+
+
+@pytest.mark.parametrize("flags", [0, 1, 2, 3])
+def test_c1_gemm(sel, flags):
+    b = gen.generate(1)
+    g = run_gpu(sel, b, flags)
+    assert_parity(g, oracle.evaluate(b), ctx=f"c1 flags={flags}")
+    assert g["counts"][0].tolist() == [24576, 532480, 532480, 8192, 524288, 2]
+
+
+@pytest.mark.parametrize("flags", [0, 2])
+def test_c2_polybench_medium(sel, flags):
+    b = gen.generate(2)
+    g = run_gpu(sel, b, flags)
+    ref = oracle.evaluate(b)
+    assert_parity(g, ref, ctx="c2")
+    st = g["stats"]
+    assert st["n_candidates"] == 108 and st["n_problems"] == 27      # 4 device sets share counts
+    assert st["wa_analysed"] * 4 == st["wa_covered"] == int(ref["W"].sum())
+
+
+def test_c2_split_api_matches_fused(sel):
+    b = gen.generate(2)
+    f = run_gpu(sel, b)
+    s = run_gpu(sel, b, api="split")
+    for k in ("counts", "status", "decision", "cycles", "t_gpu"):
+        assert np.array_equal(f[k], s[k]), k
+
+
+def test_c3_stride_offset_sweep(sel):
+    b = gen.generate(3)
+    g = run_gpu(sel, b)
+    ref = oracle.evaluate(b)
+    assert_parity(g, ref, ctx="c3")
+    # one-warp candidates (P = 32) against the closed form directly
+    acc = b.accesses[b.nests["access_off"]]
+    sb = np.abs(acc["c_par"][:, 0])
+    P = b.nests["P0"].astype(np.int64)
+    first = np.where(acc["c_par"][:, 0] < 0, acc["base"] + acc["c_par"][:, 0] * (P - 1), acc["base"])
+    o = first % 128
+    closed = np.where(sb >= 128, 32, (o + 31 * sb) // 128 - o // 128 + 1)
+    one = P == 32
+    assert one.sum() > 100
+    assert (g["counts"][one, 1].astype(np.int64) == closed[one]).all()
+
+
+def test_c4_reduced_parallel_extent(sel):
+    """c4's 24 shapes x 8 launches (B = 48, 128, 200, 1024) with the parallel
+    extent reduced to 2^14 so the oracle finishes in seconds."""
+    b = gen.generate(4)
+    nests = b.nests.copy()
+    nests["P0"] = 1 << 14
+    bb = gen.Batch(b.cands, nests, b.accesses, b.launches, b.devices)
+    for flags in (0, 1):
+        assert_parity(run_gpu(sel, bb, flags), oracle.evaluate(bb), ctx=f"c4-reduced flags={flags}")
+
+
+def test_c4_full_size_sampled(sel):
+    """Full c4 (P = 2^24) in the bench configuration; the oracle recomputes a
+    sample of candidates one by one (cheapest shapes, all 8 launches)."""
+    b = gen.generate(4)
+    g = run_gpu(sel, b)
+    names = gen.shape_names()
+    pick = [s * 8 + l for s in (names.index("mvt.1"), names.index("cov.reduce")) for l in range(8)]
+    ref = oracle.evaluate(b.select(pick))
+    sub = {k: (v[pick] if isinstance(v, np.ndarray) else v) for k, v in g.items()}
+    assert_parity(sub, ref, ctx="c4 full sampled")
+    assert (g["status"] == 0).all()
+
+
+def test_c5_full_sweep_sampled(sel):
+    """The 10^8-candidate sweep on one GPU, launched exactly as bench.py does;
+    a deterministic sample is recomputed by the oracle."""
+    b = gen.generate(5)
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
+    cands = sel._as_bytes_tensor(b.cands, "candidate")
+    r = ev.evaluate(cands, want_counts=True)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(5)
+    pick = np.unique(np.concatenate([rng.integers(0, len(b), 300), np.arange(0, len(b), len(b) // 100),
+                                     [len(b) - 1]]))
+    idx = torch.from_numpy(pick).cuda()
+    g = {k: v[idx].cpu().numpy() for k, v in r.items()}
+    g["counts"] = g["counts"].astype(np.uint64)
+    ref = oracle.evaluate(b.select(pick))
+    assert_parity(g, ref, exact_cycles=False, ctx="c5 sampled")
+    st = ev.stats()
+    assert st["n_candidates"] == 10 ** 8 and st["n_invalid"] == 0
+    # sharing: 3 B classes (32 | B, 48, 200) per (kernel, z) group of 32 candidates
+    assert st["n_problems"] == 3 * (10 ** 8 // 32)
+    assert (r["status"] == 0).all().item()
+
+
+def _random_batch(seed, n):
+    import test_oracle_counts as T
+    rnd = random.Random(seed)
+    nests = [T.random_nest(rnd) for _ in range(n)]
+    launches = np.zeros(len(nests), gen.LAUNCH_DTYPE)
+    items = []
+    for i, nn in enumerate(nests):
+        launches[i] = (nn["B"], nn["gmax"], rnd.choice([0, 32, 64]), 0)
+        items.append(dict(P0=nn["P0"], P1=nn["P1"], par_dims=nn["par_dims"], trip=nn["trip"], depth=len(nn["trip"]),
+                          comp=[rnd.random() * 4 for _ in range(4)], launch=i, device=rnd.randrange(4),
+                          cpu_cycles=10 ** rnd.uniform(3, 7), bytes_h2d=rnd.randrange(10 ** 6),
+                          accesses=[gen.make_access(base=a["base"], c_par=a["c_par"], c_inner=a["c_inner"],
+                                                    elem_bytes=a["elem"], depth=a["depth"]) for a in nn["acc"]]))
+    return gen.custom_batch(items, launches_=launches)
+
+
+@pytest.mark.parametrize("flags", [0, 1, 2])
+def test_random_tiny_nests(sel, flags):
+    """Random tiny nests: partial warps, B not a multiple of 32, #OMP_Rep > 1,
+    collapse(2) with wrapping lanes, negative and zero strides, zero trips,
+    empty iteration spaces, every element size."""
+    b = _random_batch(77 + flags, 3000)
+    assert_parity(run_gpu(sel, b, flags), oracle.evaluate(b), ctx=f"random flags={flags}")
+
+
+def test_invalid_and_edge_candidates(sel):
+    import test_oracle_model as M
+    base = M.BASE
+    a_ok = gen.make_access(base=base, c_par=(4,), elem_bytes=4, depth=0)
+    items = [
+        dict(P0=100, trip=[], accesses=[a_ok]),
+        dict(P0=100, trip=[], accesses=[a_ok], device=9),                    # V1
+        dict(P0=100, trip=[], accesses=[a_ok], cpu_hz=0.0),                  # V1
+        dict(P0=100, trip=[], accesses=[a_ok], launch=1),                    # V2 B = 0
+        dict(P0=100, trip=[], accesses=[a_ok], launch=2),                    # V2 B = 2048
+        dict(P0=100, trip=[], accesses=[a_ok], par_dims=3),                  # V3
+        dict(P0=100, P1=3, trip=[], accesses=[a_ok]),                        # V3
+        dict(P0=1 << 40, trip=[], accesses=[a_ok]),                          # V4
+        dict(P0=100, trip=[], accesses=[gen.make_access(base=base, c_par=(4,), elem_bytes=3)]),          # V5
+        dict(P0=100, trip=[], accesses=[gen.make_access(base=base + 4, c_par=(8,), elem_bytes=8)]),      # V5
+        dict(P0=100, trip=[], accesses=[gen.make_access(base=1 << 61, c_par=(1 << 56,), elem_bytes=4)]),  # V6
+        dict(P0=0, trip=[4], accesses=[gen.make_access(base=base, c_par=(4,), c_inner=(4,), elem_bytes=4, depth=1)]),
+        dict(P0=1000, trip=[], accesses=[]),                                 # W = 0 (R22)
+        dict(P0=100, trip=[0], accesses=[gen.make_access(base=base, c_par=(4,), c_inner=(4,), elem_bytes=4, depth=1)]),
+        dict(P0=100, trip=[gen.TRIP_UNKNOWN], accesses=[gen.make_access(base=base, c_par=(4,), c_inner=(4,),
+                                                                        elem_bytes=4, depth=1)]),
+        dict(P0=100, trip=[], accesses=[a_ok], launch=3),                    # V7: zero occupancy
+    ]
+    launches = np.zeros(4, gen.LAUNCH_DTYPE)
+    launches[0] = (64, 65535, 0, 0)
+    launches[1] = (0, 65535, 0, 0)
+    launches[2] = (2048, 65535, 0, 0)
+    launches[3] = (1024, 65535, 255, 0)
+    b = gen.custom_batch(items, launches_=launches)
+    ref = oracle.evaluate(b)
+    assert list(ref["status"]) == [0, 1, 1, 1, 1, 1, 1, 2, 1, 1, 2, 0, 0, 0, 0, 3]
+    for flags in (0, 1, 2):
+        g = run_gpu(sel, b, flags)
+        assert_parity(g, ref, ctx=f"edge flags={flags}")
+        assert (g["decision"][ref["status"] != 0] == 0xFF).all()
+
+
+def test_empty_batch_and_errors(sel):
+    b = gen.generate(1)
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), 4)
+    empty = torch.empty(0, dtype=torch.uint8, device="cuda")
+    r = ev.evaluate(empty)
+    assert r["decision"].numel() == 0
+    small_ws = torch.empty(256, dtype=torch.uint8, device="cuda")
+    cands = sel._as_bytes_tensor(b.cands, "candidate")
+    with pytest.raises(sel.SelError):
+        sel.evaluate(cands, ev.tables, small_ws)
+
+
+def test_deterministic_and_grid_independent(sel):
+    b = gen.generate(2)
+    g1 = run_gpu(sel, b)
+    g2 = run_gpu(sel, b)
+    for k in ("counts", "status", "decision", "cycles", "t_gpu"):
+        assert np.array_equal(g1[k], g2[k]), k
+    # reversing candidate order permutes the outputs and nothing else
+    rev = gen.Batch(b.cands[::-1].copy(), b.nests, b.accesses, b.launches, b.devices)
+    g3 = run_gpu(sel, rev)
+    for k in ("counts", "status", "decision", "cycles"):
+        assert np.array_equal(g1[k], g3[k][::-1]), k
+
+
+def test_near_tie_decisions(sel):
+    """cpu_cycles set to T_gpu * cpu_hz and +-1 ulp around it: both sides agree
+    (ties go to the CPU, R21)."""
+    b = gen.generate(2)
+    ref = oracle.evaluate(b)
+    c = b.cands.copy()
+    c["cpu_hz"] = 1.0
+    reps = []
+    for d in (-np.inf, 0, np.inf):
+        cc = c.copy()
+        cc["cpu_cycles"] = ref["t_gpu"] if d == 0 else np.nextafter(ref["t_gpu"], d)
+        reps.append(cc)
+    bt = gen.Batch(np.concatenate(reps), b.nests, b.accesses, b.launches, b.devices)
+    g = run_gpu(sel, bt)
+    r2 = oracle.evaluate(bt)
+    assert_parity(g, r2, ctx="ties")
+    n = len(b)
+    assert (g["decision"][:2 * n] == 0).all() and (g["decision"][2 * n:] == 1).all()

@@ -179,6 +179,13 @@ def profile_read():
     return ms.value, k.value
 
 
+def int_peak(mode: int = 2) -> float:
+    """Measured INT32 lane-ops/s (mode 0 ALU pipe, 1 FMA pipe, 2 both)."""
+    v = ctypes.c_double()
+    _lib.check(_lib.lib().sel_int_peak(mode, ctypes.byref(v)))
+    return v.value
+
+
 def kernel_launches() -> int:
     return int(_lib.lib().sel_kernel_launches())
 

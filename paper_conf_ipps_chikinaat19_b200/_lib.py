@@ -101,6 +101,7 @@ def lib():
         L.sel_profile_enable.argtypes = [ctypes.c_int]
         L.sel_profile_read.argtypes = [ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64)]
         L.sel_kernel_launches.restype = u64
+        L.sel_int_peak.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_double)]
         L.sel_last_error.restype = ctypes.c_char_p
         L.sel_version.restype = ctypes.c_char_p
         L.sel_sizeof.restype = sz
@@ -121,5 +122,5 @@ def check(rc: int):
 
 EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions",
             "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_read_stats",
-            "sel_profile_enable", "sel_profile_read", "sel_kernel_launches", "sel_last_error",
+            "sel_profile_enable", "sel_profile_read", "sel_kernel_launches", "sel_int_peak", "sel_last_error",
             "sel_version", "sel_sizeof", "sel_offsetof")

@@ -13,9 +13,10 @@
 // flattened WA index space (problem, access, warp-rep, inner tuple) from an
 // atomic counter, so a 16-WA nest and a 10^9-WA nest are balanced alike; a
 // warp decodes its chunk start once (32-ary search over the problem prefix,
-// one div/mod) and then walks with odometer steps.
+// one div/mod) and then walks with odometer steps.  A chunk holds at most
+// 2^20 WAs, so every accumulator is 32-bit until the per-chunk flush.
 //
-// Two exact counting primitives (DESIGN.md "Count kernel"):
+// Two exact counting primitives (DESIGN.md §7):
 //  * RESIDUE (default).  Per warp-rep the lane addresses A_l are fixed and
 //    every inner iteration adds the same offset D to all of them, so their
 //    sorted order and the gaps d_l between sorted neighbours are fixed.  Then
@@ -26,7 +27,7 @@
 //    traffic.  1-D parallel accesses are monotone across lanes (no sort);
 //    collapse(2) accesses are sorted once per warp-rep with a shuffle
 //    bitonic network.  lines = 1 + #flags; coalesced (tmin = 1) <=> no flag
-//    (__any_sync); tmin > 1 uses __ballot_sync/__popc.
+//    (vote.any); tmin > 1 uses vote.ballot + popc.
 //  * MATCH (SEL_F_MATCH_ANY).  The north star's literal primitive: full
 //    64-bit lane addresses, __match_any_sync on (addr >> 7) and (addr >> 5),
 //    first-occurrence flags, __ballot_sync/__popc.
@@ -34,6 +35,8 @@
 #include "sel_internal.h"
 
 namespace sel {
+
+constexpr uint64_t kMaxChunk = 1ull << 20;   // WAs per chunk: keeps all accumulators 32-bit
 
 struct CountArgs {
     const sel_nest* nests;
@@ -46,13 +49,15 @@ struct CountArgs {
     WsHeader* hdr;
 };
 
-// per-warp accumulators for the problem being counted
+// Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
+//  RESIDUE: L = W + sum(lf_lane) + lk ; S = W + sum(sf_lane) ;
+//           U = (W1 - C1) + sum(lf_lane) + (W2 - C2) + uk
+//  (lf_lane only from tmin = 1 accesses, whose coalesced WAs have no flag;
+//   lk / uk: uniform flag counts of tmin > 1 accesses / of their uncoalesced WAs)
+//  MATCH:   L, S, U accumulated directly (uniform).
 struct Acc {
-    uint32_t LfA;        // per lane: line flags of tmin = 1 accesses
-    uint32_t Sf;         // per lane: sector flags of all accesses (RESIDUE)
-    uint64_t W1, C1;     // uniform: WAs / coalesced WAs of tmin = 1 accesses
-    uint64_t W2, C2, L2, U2;   // uniform: tmin > 1 accesses (lines counted exactly)
-    uint64_t Lm, Sm;     // uniform: MATCH path totals
+    uint32_t lf, sf;                 // per lane
+    uint32_t W1, C1, W2, C2, lk, uk; // uniform
 };
 
 __device__ __forceinline__ unsigned lanemask_lt() {
@@ -95,72 +100,70 @@ __device__ __forceinline__ int64_t bitonic_sort_warp(int64_t key, int lane) {
     return key;
 }
 
-// lane address of warp-rep m, without the inner-loop part; sets n (active lanes)
-__device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B,
-                                                uint64_t m, int lane, int* n_out) {
-    uint64_t p0;
-    uint32_t n;
-    if ((B & 31u) == 0) {
-        p0 = m * 32;
-        n = uint32_t(umin64(32, P - p0));
-    } else {
-        const uint32_t wpb = (B + 31) >> 5;
-        const uint64_t kb = m / wpb;
-        const uint32_t w = uint32_t(m - kb * wpb);
-        p0 = kb * B + 32ull * w;
-        n = uint32_t(umin64(umin64(32, B - 32 * w), P - p0));
-    }
-    *n_out = int(n);
-    const uint64_t p = p0 + uint64_t(lane < int(n) ? lane : 0);
-    if (nest.par_dims == 1) return a.base + a.c_par[0] * int64_t(p);
-    return a.base + a.c_par[0] * int64_t(p / nest.P1) + a.c_par[1] * int64_t(p % nest.P1);
-}
-
-// ----------------------------------------------------------- RESIDUE loops
-template <bool T1>
-__device__ __forceinline__ void hot_residue(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint64_t len,
-                                            int tmin, Acc& acc) {
-    uint32_t lf = 0, sf = 0, c = 0;
-    uint64_t l2 = 0, u2 = 0;
+// ------------------------------------------------------------- hot loops
+// RESIDUE, tmin = 1 (elements of 1, 2, 4 bytes): per WA and lane
+//   line flag  y < dl ; sector flag (y << 2) < ds ; coalesced <=> no line flag.
+__device__ __forceinline__ void hot_t1(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
+                                       Acc& a) {
+    uint32_t lf = a.lf, sf = a.sf, c = a.C1;
 #pragma unroll 4
-    for (uint64_t i = 0; i < len; i++) {
-        const bool fl = y < dl;
-        const bool fs = (y << 2) < ds;
-        sf += fs;
-        if (T1) {
-            lf += fl;
-            c += !__any_sync(kFull, fl);
-        } else {
-            const int lines = __popc(__ballot_sync(kFull, fl)) + 1;
-            const bool coal = lines <= tmin;
-            c += coal;
-            l2 += lines;
-            u2 += coal ? 0 : lines;
-        }
+    for (uint32_t i = 0; i < len; i++) {
+        const uint32_t z = y << 2;
+        asm("{\n\t.reg .pred pl, ps, pa;\n\t"
+            "setp.lt.u32 pl, %3, %5;\n\t"
+            "setp.lt.u32 ps, %4, %6;\n\t"
+            "@pl add.u32 %0, %0, 1;\n\t"
+            "@ps add.u32 %1, %1, 1;\n\t"
+            "vote.sync.any.pred pa, pl, 0xffffffff;\n\t"
+            "@!pa add.u32 %2, %2, 1;\n\t}"
+            : "+r"(lf), "+r"(sf), "+r"(c)
+            : "r"(y), "r"(z), "r"(dl), "r"(ds));
         y += step;
     }
-    acc.Sf += sf;
-    if (T1) {
-        acc.LfA += lf;
-        acc.W1 += len;
-        acc.C1 += c;
-    } else {
-        acc.W2 += len;
-        acc.C2 += c;
-        acc.L2 += l2;
-        acc.U2 += u2;
-    }
+    a.lf = lf;
+    a.sf = sf;
+    a.C1 = c;
+    a.W1 += len;
 }
 
-template <bool T1>
-__device__ __forceinline__ void hot_match(int64_t addr, int64_t step, uint64_t len, int tmin, Acc& acc) {
+// RESIDUE, tmin = 2 or 4 (8 or 16 byte elements): the number of line flags
+// decides the class, so the flags are counted with ballot + popc.
+__device__ __forceinline__ void hot_t2(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
+                                       uint32_t tm1, Acc& a) {
+    uint32_t sf = a.sf, c = a.C2, lk = a.lk, uk = a.uk;
+#pragma unroll 4
+    for (uint32_t i = 0; i < len; i++) {
+        const uint32_t z = y << 2;
+        asm("{\n\t.reg .pred pl, ps, pc;\n\t.reg .b32 b, k;\n\t"
+            "setp.lt.u32 pl, %4, %6;\n\t"
+            "setp.lt.u32 ps, %5, %7;\n\t"
+            "@ps add.u32 %0, %0, 1;\n\t"
+            "vote.sync.ballot.b32 b, pl, 0xffffffff;\n\t"
+            "popc.b32 k, b;\n\t"
+            "add.u32 %2, %2, k;\n\t"
+            "setp.le.u32 pc, k, %8;\n\t"
+            "@pc add.u32 %1, %1, 1;\n\t"
+            "@!pc add.u32 %3, %3, k;\n\t}"
+            : "+r"(sf), "+r"(c), "+r"(lk), "+r"(uk)
+            : "r"(y), "r"(z), "r"(dl), "r"(ds), "r"(tm1));
+        y += step;
+    }
+    a.sf = sf;
+    a.C2 = c;
+    a.lk = lk;
+    a.uk = uk;
+    a.W2 += len;
+}
+
+// MATCH: literal __match_any_sync expansion over 64-bit lane addresses.
+__device__ __forceinline__ void hot_match(int64_t addr, int64_t step, uint32_t len, uint32_t tmin, Acc& a) {
     const unsigned lt = lanemask_lt();
-    uint64_t L = 0, S = 0, C = 0, U = 0;
-    for (uint64_t i = 0; i < len; i++) {
+    uint32_t L = 0, S = 0, C = 0, U = 0;
+    for (uint32_t i = 0; i < len; i++) {
         const unsigned ml = __match_any_sync(kFull, (unsigned long long)(addr >> 7));
         const unsigned ms = __match_any_sync(kFull, (unsigned long long)(addr >> 5));
-        const int lines = __popc(__ballot_sync(kFull, (ml & lt) == 0));
-        const int sectors = __popc(__ballot_sync(kFull, (ms & lt) == 0));
+        const uint32_t lines = __popc(__ballot_sync(kFull, (ml & lt) == 0));
+        const uint32_t sectors = __popc(__ballot_sync(kFull, (ms & lt) == 0));
         const bool coal = lines <= tmin;
         L += lines;
         S += sectors;
@@ -168,111 +171,153 @@ __device__ __forceinline__ void hot_match(int64_t addr, int64_t step, uint64_t l
         U += coal ? 0 : lines;
         addr += step;
     }
-    acc.Lm += L;
-    acc.Sm += S;
-    acc.W1 += len;
-    acc.C1 += C;
-    acc.U2 += U;
+    a.lk += L;      // MATCH: lk = lines, uk = uncoalesced lines, sf(lane 0) = sectors
+    a.uk += U;
+    a.sf += S;
+    a.C1 += C;
+    a.W1 += len;
 }
 
-// Count WAs [off, off + cnt) of access `a` of a problem (instance order:
-// warp-rep m, then inner tuple with the last inner loop fastest).
-template <bool MATCH>
-__device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B,
-                             const uint64_t* T, uint64_t Mk, uint64_t off, uint64_t cnt, int lane, Acc& acc) {
-    const int depth = a.depth;
-    const int tmin = (32 * int(a.elem_bytes) + 127) / 128;        // R11
+// --------------------------------------------------------- warp iterator
+// Enumerates the active warps of a problem (R8, R9): block k covers
+// iterations [kB, kB + B) and holds ceil(B/32) warps, the last one partial
+// when 32 does not divide B; warps past P are skipped (WR counts the rest).
+struct WarpIter {
+    uint64_t p0;        // first iteration of the warp
+    uint64_t blk_end;   // end of the current block's iterations
+    uint32_t n;         // active lanes
+};
+
+__device__ __forceinline__ void warp_seek(WarpIter& it, uint64_t m, uint64_t P, uint32_t B) {
+    if ((B & 31u) == 0) {
+        it.p0 = m * 32;
+        it.blk_end = ~0ull;
+    } else {
+        const uint32_t wpb = (B + 31) >> 5;
+        const uint64_t kb = m / wpb;
+        const uint32_t w = uint32_t(m - kb * wpb);
+        it.p0 = kb * B + 32ull * w;
+        it.blk_end = (kb + 1) * B;
+    }
+    uint64_t e = it.p0 + 32;
+    if (e > it.blk_end) e = it.blk_end;
+    if (e > P) e = P;
+    it.n = uint32_t(e - it.p0);
+}
+
+__device__ __forceinline__ void warp_next(WarpIter& it, uint64_t P, uint32_t B) {
+    uint64_t p = it.p0 + 32;
+    if (p >= it.blk_end) {               // next block (only when 32 does not divide B)
+        p = it.blk_end;
+        it.blk_end += B;
+    }
+    it.p0 = p;
+    uint64_t e = p + 32;
+    if (e > it.blk_end) e = it.blk_end;
+    if (e > P) e = P;
+    it.n = uint32_t(e - p);
+}
+
+// lane address of the current warp without the inner-loop part (a2, R25)
+__device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_access& a, const WarpIter& it,
+                                                int lane) {
+    const uint64_t p = it.p0 + uint64_t(lane < int(it.n) ? lane : 0);
+    if (nest.par_dims == 1) return a.base + a.c_par[0] * int64_t(p);
+    return a.base + a.c_par[0] * int64_t(p / nest.P1) + a.c_par[1] * int64_t(p % nest.P1);
+}
+
+// ------------------------------------------------------------- per access
+// Count WAs [off, off + cnt) of access `a` (instance order: warp-rep, then
+// inner tuple with the last inner loop fastest).  DEPTH = a.depth.
+template <bool MATCH, int DEPTH, bool T1>
+__device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B, uint64_t T0,
+                             uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t cnt, int lane, Acc& acc) {
+    const uint32_t tmin = (32u * a.elem_bytes + 127u) / 128u;       // R11
+    const uint64_t Tl = DEPTH == 1 ? T0 : DEPTH == 2 ? T1 : DEPTH == 3 ? T2 : 1;
+    const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
     uint64_t m = off / Mk;
     uint64_t tt = off - m * Mk;
-    uint64_t idx[3] = {0, 0, 0};
-    {
-        uint64_t r = tt;
-        for (int j = depth - 1; j >= 0; j--) {
-            idx[j] = r % T[j];
-            r /= T[j];
-        }
-    }
-    const int64_t c_last = depth ? a.c_inner[depth - 1] : 0;
-    const uint64_t T_last = depth ? T[depth - 1] : 1;
+    // inner indices, last fastest
+    uint64_t i0 = 0, i1 = 0, i2 = 0;
+    if (DEPTH == 1) { i0 = tt; }
+    if (DEPTH == 2) { i1 = tt % T1; i0 = tt / T1; }
+    if (DEPTH == 3) { i2 = tt % T2; const uint64_t r = tt / T2; i1 = r % T1; i0 = r / T1; }
+    WarpIter it;
+    warp_seek(it, m, P, B);
     while (cnt > 0) {
-        int n;
-        const int64_t A = lane_address(nest, a, P, B, m, lane, &n);
-        // per-warp-rep setup
+        const int64_t A = lane_address(nest, a, it, lane);
         uint32_t u_low = 0, dl = 0, ds = 0;
         int64_t Am = A;
         if (!MATCH) {
             int64_t upper;
             uint64_t gap;
-            bool has;
             if (nest.par_dims == 1) {
                 const int64_t c0 = a.c_par[0];
-                upper = A + (c0 < 0 ? -c0 : 0);     // larger address of the pair (l-1, l)
+                upper = A + (c0 < 0 ? -c0 : 0);     // larger address of the lane pair (l-1, l)
                 gap = uabs(c0);
-                has = lane >= 1 && lane < n;
             } else {
-                const int64_t key = bitonic_sort_warp(lane < n ? A : INT64_MAX, lane);
+                const int64_t key = bitonic_sort_warp(lane < int(it.n) ? A : INT64_MAX, lane);
                 const int64_t prev = __shfl_up_sync(kFull, key, 1);
                 upper = key;
                 gap = uint64_t(key - prev);
-                has = lane >= 1 && lane < n;
             }
+            const bool has = lane >= 1 && lane < int(it.n);
             u_low = uint32_t(upper);
             dl = has ? (gap >= 128 ? 0xffffffffu : uint32_t(gap) << 25) : 0u;
             ds = has ? (gap >= 32 ? 0xffffffffu : uint32_t(gap) << 27) : 0u;
         } else {
             const int64_t a0 = __shfl_sync(kFull, A, 0);
-            Am = lane < n ? A : a0;                 // inactive lanes duplicate lane 0
+            Am = lane < int(it.n) ? A : a0;         // inactive lanes duplicate lane 0
         }
-        const uint64_t here = umin64(Mk - tt, cnt);
-        uint64_t left = here;
+        // rows of the last inner loop within this warp-rep
+        const uint64_t here64 = umin64(Mk - tt, cnt);
+        uint32_t left = uint32_t(here64);
         while (left > 0) {
             int64_t D = 0;
-            for (int j = 0; j < depth; j++) D += a.c_inner[j] * int64_t(idx[j]);
-            const uint64_t i_last = depth ? idx[depth - 1] : 0;
-            const uint64_t len = umin64(T_last - i_last, left);
+            if (DEPTH >= 1) D += a.c_inner[0] * int64_t(i0);
+            if (DEPTH >= 2) D += a.c_inner[1] * int64_t(i1);
+            if (DEPTH >= 3) D += a.c_inner[2] * int64_t(i2);
+            const uint64_t il = DEPTH == 1 ? i0 : DEPTH == 2 ? i1 : DEPTH == 3 ? i2 : 0;
+            const uint32_t len = uint32_t(umin64(Tl - il, left));
             if (MATCH) {
-                if (tmin == 1) hot_match<true>(Am + D, c_last, len, tmin, acc);
-                else hot_match<false>(Am + D, c_last, len, tmin, acc);
+                hot_match(Am + D, cl, len, tmin, acc);
             } else {
                 const uint32_t y = (u_low + uint32_t(uint64_t(D))) << 25;
-                const uint32_t step = uint32_t(uint64_t(c_last)) << 25;
-                if (tmin == 1) hot_residue<true>(y, step, dl, ds, len, tmin, acc);
-                else hot_residue<false>(y, step, dl, ds, len, tmin, acc);
+                const uint32_t step = uint32_t(uint64_t(cl)) << 25;
+                if (T1) hot_t1(y, step, dl, ds, len, acc);
+                else hot_t2(y, step, dl, ds, len, tmin - 1, acc);
             }
             left -= len;
-            // odometer carry
-            if (depth) {
-                idx[depth - 1] += len;
-                int j = depth - 1;
-                while (j >= 0 && idx[j] >= T[j]) {
-                    idx[j] = 0;
-                    if (j > 0) idx[j - 1] += 1;
-                    j--;
-                }
+            // odometer carry (registers only)
+            if (DEPTH == 1) { i0 += len; if (i0 >= T0) i0 = 0; }
+            if (DEPTH == 2) { i1 += len; if (i1 >= T1) { i1 = 0; if (++i0 >= T0) i0 = 0; } }
+            if (DEPTH == 3) {
+                i2 += len;
+                if (i2 >= T2) { i2 = 0; if (++i1 >= T1) { i1 = 0; if (++i0 >= T0) i0 = 0; } }
             }
         }
-        cnt -= here;
-        m += 1;
+        cnt -= uint32_t(here64);
         tt = 0;
+        if (cnt > 0) warp_next(it, P, B);
     }
 }
 
 template <bool MATCH>
 __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
-    const uint32_t sumLfA = __reduce_add_sync(kFull, acc.LfA);
-    const uint32_t sumSf = __reduce_add_sync(kFull, acc.Sf);
-    const uint64_t W = acc.W1 + acc.W2;
+    const uint32_t W = acc.W1 + acc.W2;
     uint64_t L, S, C, U;
     if (MATCH) {
-        L = acc.Lm;
-        S = acc.Sm;
+        L = acc.lk;
+        S = acc.sf;
         C = acc.C1;
-        U = acc.U2;
+        U = acc.uk;
     } else {
-        L = acc.W1 + sumLfA + acc.L2;
-        S = W + sumSf;
-        C = acc.C1 + acc.C2;
-        U = (acc.W1 - acc.C1) + sumLfA + acc.U2;
+        const uint64_t slf = __reduce_add_sync(kFull, acc.lf);
+        const uint64_t ssf = __reduce_add_sync(kFull, acc.sf);
+        L = uint64_t(W) + slf + acc.lk;
+        S = uint64_t(W) + ssf;
+        C = uint64_t(acc.C1) + acc.C2;
+        U = uint64_t(acc.W1 - acc.C1) + slf + uint64_t(acc.W2 - acc.C2) + acc.uk;
     }
     if (W && lane < 5) {
         const uint64_t v = lane == 0 ? W : lane == 1 ? L : lane == 2 ? S : lane == 3 ? C : U;
@@ -282,25 +327,46 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
 }
 
 template <bool MATCH>
-__device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint64_t take, int lane) {
+__device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane) {
     const sel_nest nest = a.nests[a.prob_nest[q]];
     const uint32_t B = a.prob_B[q];
     const uint64_t WR = a.prob_WR[q];
     const uint64_t P = nest.P0 * nest.P1;
-    uint64_t T[3];
-    for (int j = 0; j < 3; j++) T[j] = eff_trip(nest.trip[j]);
+    const uint64_t T0 = eff_trip(nest.trip[0]), T1 = eff_trip(nest.trip[1]), T2 = eff_trip(nest.trip[2]);
     Acc acc{};
     for (uint32_t k = 0; k < nest.n_access && take > 0; k++) {
         const sel_access ac = a.acc[nest.access_off + k];
-        uint64_t Mk = 1;
-        for (int j = 0; j < ac.depth; j++) Mk *= T[j];
+        const int d = ac.depth;
+        const uint64_t Mk = d == 0 ? 1 : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
         const uint64_t Wk = WR * Mk;
         if (off >= Wk) {
             off -= Wk;
             continue;
         }
-        const uint64_t t = umin64(Wk - off, take);
-        count_access<MATCH>(nest, ac, P, B, T, Mk, off, t, lane, acc);
+        const uint32_t t = uint32_t(umin64(Wk - off, take));
+        const bool t1 = ac.elem_bytes <= 4;                     // tmin = ceil(32 e / 128) = 1
+        if (MATCH) {
+            switch (d) {
+            case 0: count_access<true, 0, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 1: count_access<true, 1, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 2: count_access<true, 2, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            default: count_access<true, 3, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            }
+        } else if (t1) {
+            switch (d) {
+            case 0: count_access<false, 0, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 1: count_access<false, 1, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 2: count_access<false, 2, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            default: count_access<false, 3, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            }
+        } else {
+            switch (d) {
+            case 0: count_access<false, 0, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 1: count_access<false, 1, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            case 2: count_access<false, 2, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            default: count_access<false, 3, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
+            }
+        }
         take -= t;
         off = 0;
     }
@@ -308,7 +374,7 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
 }
 
 template <bool MATCH>
-__global__ void __launch_bounds__(256, 4) k_count(CountArgs a) {
+__global__ void __launch_bounds__(256, 3) k_count(CountArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;
@@ -316,14 +382,14 @@ __global__ void __launch_bounds__(256, 4) k_count(CountArgs a) {
     if (total == 0) return;
     const uint64_t nwarps = uint64_t(gridDim.x) * (blockDim.x >> 5);
     uint64_t ch = total / (nwarps * 16);
-    ch = ch < 256 ? 256 : (ch > (1ull << 20) ? (1ull << 20) : ch);
+    ch = ch < 256 ? 256 : (ch > kMaxChunk ? kMaxChunk : ch);
     for (;;) {
         unsigned long long chunk = 0;
         if (lane == 0) chunk = atomicAdd(&a.hdr->chunk_ctr, 1ull);
         chunk = __shfl_sync(kFull, chunk, 0);
         const uint64_t start = chunk * ch;
         if (start >= total) break;
-        uint64_t len = umin64(ch, total - start);
+        uint32_t len = uint32_t(umin64(ch, total - start));
         uint64_t q = find_problem(a.prefix, nq, start, lane);
         uint64_t off = start - a.prefix[q];
         while (len > 0) {
@@ -333,7 +399,7 @@ __global__ void __launch_bounds__(256, 4) k_count(CountArgs a) {
                 q++;
                 continue;
             }
-            const uint64_t take = umin64(Wq - off, len);
+            const uint32_t take = uint32_t(umin64(Wq - off, len));
             count_problem<MATCH>(a, q, off, take, lane);
             len -= take;
             off = 0;

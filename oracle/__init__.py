@@ -57,6 +57,7 @@ def lib():
         L.oracle_evaluate.argtypes = [vp, ctypes.c_int, vp, u64, vp, u64, vp, u64, vp, u64, vp,
                                       ctypes.c_int]
         L.oracle_model.argtypes = [vp, vp, vp, vp, vp, vp]
+        L.oracle_select_launch.argtypes = [vp, u64, vp, vp, u64, vp, vp]
         L.oracle_sizeof.restype = ctypes.c_size_t
         L.oracle_sizeof.argtypes = [ctypes.c_int]
         L.oracle_offsetof.restype = ctypes.c_size_t
@@ -104,6 +105,18 @@ def model(device, nest, accesses, launch, cand, W, L, S, C, U, WR) -> np.void:
     lib().oracle_model(dv.ctypes.data, ne.ctypes.data, ac.ctypes.data, la.ctypes.data,
                        cd.ctypes.data, r.ctypes.data)
     return r[0]
+
+
+def select_launch(group_of, t_gpu, status, n_groups):
+    """NEXT row f3: per-group argmin of t_gpu (see oracle.c)."""
+    g = np.ascontiguousarray(group_of, dtype=np.uint32)
+    t = np.ascontiguousarray(t_gpu, dtype=np.float64)
+    s = np.ascontiguousarray(status, dtype=np.uint8)
+    best = np.zeros(n_groups, np.uint32)
+    val = np.zeros(n_groups, np.float64)
+    lib().oracle_select_launch(g.ctypes.data, len(g), t.ctypes.data, s.ctypes.data, n_groups, best.ctypes.data,
+                               val.ctypes.data)
+    return best, val
 
 
 def layout(which: int):

@@ -409,3 +409,20 @@ size_t oracle_offsetof(int which, int field) {
     }
     return (field >= 0 && (size_t)field < nf) ? t[field] : (size_t)-1;
 }
+
+/* -------------------------------------------------- NEXT row f3 (launch) */
+/* Launch-configuration selection ("the maximum
+ * grid-geometry selected by the runtime", P:L331 ML grid-geometry
+ * predictors whose inference is too slow): for every group g of candidates
+ * (the same nest and device under different launch configurations), the
+ * valid candidate with the smallest predicted GPU time; ties and +inf go to
+ * the lowest candidate index.  Plain definition: one ascending pass. */
+void oracle_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
+                          uint64_t n_groups, uint32_t* best, double* best_val) {
+    for (uint64_t g = 0; g < n_groups; g++) { best[g] = 0xFFFFFFFFu; best_val[g] = INFINITY; }
+    for (uint64_t c = 0; c < n; c++) {
+        uint64_t g = group_of[c];
+        if (g >= n_groups || status[c] != 0) continue;
+        if (best[g] == 0xFFFFFFFFu || t_gpu[c] < best_val[g]) { best[g] = (uint32_t)c; best_val[g] = t_gpu[c]; }
+    }
+}

@@ -82,6 +82,11 @@ int oracle_evaluate(const or_device* devs, int n_devs,
 void oracle_model(const or_device* dev, const or_nest* nest, const or_access* acc,
                   const or_launch* launch, const or_candidate* cand, or_result* r);
 
+/* NEXT row f3: per-group argmin of t_gpu over valid candidates (ties and
+ * +inf: lowest index; no valid candidate: best = 0xFFFFFFFF, +inf). */
+void oracle_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
+                          uint64_t n_groups, uint32_t* best, double* best_val);
+
 /* Layout self-description for tests/test_layout.py. */
 size_t oracle_sizeof(int which);
 size_t oracle_offsetof(int which, int field);

@@ -160,6 +160,17 @@ def evaluate(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor,
     return out
 
 
+def select_launch(group_of: torch.Tensor, t_gpu: torch.Tensor, status: torch.Tensor, n_groups: int, stream=None):
+    """sel_select_launch (NEXT row f3) -> (best uint32-as-int32[n_groups], best_t_gpu f64[n_groups])."""
+    _require_cuda(group_of, t_gpu, status)
+    n = t_gpu.numel()
+    best = torch.empty(n_groups, dtype=torch.int32, device=t_gpu.device)
+    best_t = torch.empty(n_groups, dtype=torch.float64, device=t_gpu.device)
+    _lib.check(_lib.lib().sel_select_launch(_ptr(group_of), n, _ptr(t_gpu), _ptr(status), n_groups, _ptr(best),
+                                            _ptr(best_t), _stream(stream)))
+    return best, best_t
+
+
 def read_stats(workspace: torch.Tensor, stream=None) -> dict:
     st = _lib.Stats()
     wp, _ = _ws_ptr(workspace)
@@ -198,6 +209,7 @@ sel_predict_gpu_cycles = predict_gpu_cycles
 sel_select = select
 sel_evaluate = evaluate
 sel_read_stats = read_stats
+sel_select_launch = select_launch
 
 
 class Evaluator:

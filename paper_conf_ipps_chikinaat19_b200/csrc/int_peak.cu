@@ -17,11 +17,11 @@ __global__ void __launch_bounds__(512) k_int_peak(uint32_t iters, uint32_t seed,
     for (uint32_t i = 0; i < iters; i++) {
 #pragma unroll
         for (int u = 0; u < 8; u++) {
-            if (MODE == 0 || MODE == 2) {      // ALU pipe: IADD3 / LOP3
-                asm volatile("add.u32 %0, %0, %1;" : "+r"(a0) : "r"(k));
-                asm volatile("xor.b32 %0, %0, %1;" : "+r"(a1) : "r"(k));
-                asm volatile("add.u32 %0, %0, %1;" : "+r"(a2) : "r"(k));
-                asm volatile("xor.b32 %0, %0, %1;" : "+r"(a3) : "r"(k));
+            if (MODE == 0 || MODE == 2) {      // ALU pipe: IADD3 / LOP3, mutually dependent (not foldable)
+                asm volatile("add.u32 %0, %0, %1;" : "+r"(a0) : "r"(a1));
+                asm volatile("xor.b32 %0, %0, %1;" : "+r"(a1) : "r"(a2));
+                asm volatile("add.u32 %0, %0, %1;" : "+r"(a2) : "r"(a3));
+                asm volatile("xor.b32 %0, %0, %1;" : "+r"(a3) : "r"(a0));
             }
             if (MODE == 1 || MODE == 2) {      // FMA pipe: IMAD
                 asm volatile("mad.lo.u32 %0, %0, %1, %1;" : "+r"(b0) : "r"(k));

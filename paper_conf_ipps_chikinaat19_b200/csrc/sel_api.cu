@@ -186,6 +186,17 @@ int sel_evaluate(const sel_candidate* c, uint64_t n, const sel_tables* t, uint8_
     return SEL_OK;
 }
 
+int sel_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
+                      uint64_t n_groups, uint32_t* best, double* best_t, sel_stream_t stream) {
+    if (n_groups == 0) return SEL_OK;
+    if (!best || !best_t || (n && (!group_of || !t_gpu || !status))) return fail(SEL_EINVAL, "NULL argument%s");
+    if (n >= 0xffffffffull) return fail(SEL_EINVAL, "n must be < 2^32 - 1%s");
+    cudaError_t e = launch_select_launch(group_of, n, t_gpu, status, n_groups, best, best_t,
+                                         reinterpret_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "select_launch");
+    return SEL_OK;
+}
+
 int sel_read_stats(const void* ws, sel_stats* out, sel_stream_t stream) {
     if (!ws || !out) return fail(SEL_EINVAL, "NULL argument%s");
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);

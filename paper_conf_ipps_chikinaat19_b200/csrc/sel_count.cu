@@ -50,16 +50,16 @@ struct CountArgs {
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
-//  RESIDUE: L = W + sum(lf_lane) + lk ; S = W + sum(sf_lane) ;
-//           U = (W1 - C1) + sum(lf_lane) + (W2 - C2) + uk
-//  (lf_lane only from tmin = 1 accesses, whose coalesced WAs have no flag;
-//   lk / uk: uniform flag counts of tmin > 1 accesses / of their uncoalesced WAs)
-//  MATCH:   L, S, U accumulated directly (uniform).
+//   L = W + sum_lanes(lf) + lk      S = W + sum_lanes(sf) + sk
+//   C = C                           U = (W - C) + sum_lanes(uf) + uk
+// lf / sf: per-lane line / sector flags (a lane whose line or sector differs
+// from its sorted predecessor's); uf: line flags of uncoalesced WAs.
+// lk, sk, uk: the same quantities accumulated warp-uniformly (tmin = 4 and
+// MATCH paths).
 struct Acc {
-    uint32_t lf, sf;                 // per lane
-    uint32_t W1, C1, W2, C2, lk, uk; // uniform
+    uint32_t lf, sf, uf;             // per lane
+    uint32_t W, C, lk, sk, uk;       // uniform
 };
-
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -101,58 +101,104 @@ __device__ __forceinline__ int64_t bitonic_sort_warp(int64_t key, int lane) {
 }
 
 // ------------------------------------------------------------- hot loops
-// RESIDUE, tmin = 1 (elements of 1, 2, 4 bytes): per WA and lane
-//   line flag  y < dl ; sector flag (y << 2) < ds ; coalesced <=> no line flag.
-__device__ __forceinline__ void hot_t1(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
-                                       Acc& a) {
-    uint32_t lf = a.lf, sf = a.sf, c = a.C1;
-#pragma unroll 4
-    for (uint32_t i = 0; i < len; i++) {
-        const uint32_t z = y << 2;
-        asm("{\n\t.reg .pred pl, ps, pa;\n\t"
-            "setp.lt.u32 pl, %3, %5;\n\t"
-            "setp.lt.u32 ps, %4, %6;\n\t"
-            "@pl add.u32 %0, %0, 1;\n\t"
-            "@ps add.u32 %1, %1, 1;\n\t"
-            "vote.sync.any.pred pa, pl, 0xffffffff;\n\t"
-            "@!pa add.u32 %2, %2, 1;\n\t}"
-            : "+r"(lf), "+r"(sf), "+r"(c)
-            : "r"(y), "r"(z), "r"(dl), "r"(ds));
-        y += step;
-    }
-    a.lf = lf;
-    a.sf = sf;
-    a.C1 = c;
-    a.W1 += len;
+// RESIDUE.  Per lane and WA: line flag  y < dl,  sector flag  (y << 2) < ds.
+// WAs are processed in groups of up to 32 consecutive inner iterations: each
+// lane sets bit i of m when it has a line flag in WA i of the group, so the
+// class of the 32 WAs needs one warp reduction per group instead of a vote
+// per WA (coalesced <=> lines <= tmin <=> #flags <= tmin - 1, R11):
+//   tmin = 1: uncoalesced WAs = OR over lanes of m
+//   tmin = 2: uncoalesced WAs = OR over lanes of (m & exclusive-prefix-OR of m)
+//             (bit i set <=> at least two lanes flag WA i)
+// tmin = 4 (16-byte elements) keeps a per-WA ballot + popc.
+
+// one WA of a group: bit `bit` of m, sector flag count
+__device__ __forceinline__ void wa_step(uint32_t& m, uint32_t& sf, uint32_t y, uint32_t dl, uint32_t ds,
+                                        uint32_t bit) {
+    const uint32_t z = y << 2;
+    asm("{\n\t.reg .pred pl, ps;\n\t"
+        "setp.lt.u32 pl, %2, %4;\n\t"
+        "setp.lt.u32 ps, %3, %5;\n\t"
+        "@pl or.b32 %0, %0, %6;\n\t"
+        "@ps add.u32 %1, %1, 1;\n\t}"
+        : "+r"(m), "+r"(sf)
+        : "r"(y), "r"(z), "r"(dl), "r"(ds), "r"(bit));
 }
 
-// RESIDUE, tmin = 2 or 4 (8 or 16 byte elements): the number of line flags
-// decides the class, so the flags are counted with ballot + popc.
-__device__ __forceinline__ void hot_t2(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
-                                       uint32_t tm1, Acc& a) {
-    uint32_t sf = a.sf, c = a.C2, lk = a.lk, uk = a.uk;
-#pragma unroll 4
+template <int TC>
+__device__ __forceinline__ void group_end(uint32_t m, uint32_t g, Acc& a) {
+    uint32_t unc;
+    if (TC == 1) {
+        unc = __reduce_or_sync(kFull, m);
+    } else {
+        uint32_t x = m;                                   // inclusive prefix OR over lanes
+        const int lane = threadIdx.x & 31;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(kFull, x, o);
+            if (lane >= o) x |= t;
+        }
+        uint32_t ex = __shfl_up_sync(kFull, x, 1);
+        if (lane == 0) ex = 0;
+        unc = __reduce_or_sync(kFull, m & ex);
+    }
+    a.lf += __popc(m);
+    a.uf += __popc(m & unc);
+    a.C += g - __popc(unc);
+    a.W += g;
+}
+
+template <int TC>
+__device__ __forceinline__ void hot_row(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
+                                        Acc& a) {
+    // four independent accumulator chains (ILP): WA i of a group uses chain i & 3
+    uint32_t s0 = 0, s1 = 0, s2 = 0, s3 = 0;
+    while (len >= 32) {                                   // full groups: bits are immediates
+        uint32_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
+#pragma unroll
+        for (int i = 0; i < 32; i += 4) {
+            wa_step(m0, s0, y + uint32_t(i) * step, dl, ds, 1u << i);
+            wa_step(m1, s1, y + uint32_t(i + 1) * step, dl, ds, 2u << i);
+            wa_step(m2, s2, y + uint32_t(i + 2) * step, dl, ds, 4u << i);
+            wa_step(m3, s3, y + uint32_t(i + 3) * step, dl, ds, 8u << i);
+        }
+        y += 32u * step;
+        group_end<TC>((m0 | m1) | (m2 | m3), 32, a);
+        len -= 32;
+    }
+    if (len) {                                            // partial group
+        uint32_t m0 = 0, m1 = 0, bit = 1;
+        uint32_t i = 0;
+        for (; i + 2 <= len; i += 2) {
+            wa_step(m0, s0, y, dl, ds, bit);
+            wa_step(m1, s1, y + step, dl, ds, bit << 1);
+            bit <<= 2;
+            y += 2u * step;
+        }
+        if (i < len) wa_step(m0, s2, y, dl, ds, bit);
+        group_end<TC>(m0 | m1, len, a);
+    }
+    a.sf += (s0 + s1) + (s2 + s3);
+}
+
+// tmin = 4: per-WA ballot + popc
+__device__ __forceinline__ void hot_row_t4(uint32_t y, uint32_t step, uint32_t dl, uint32_t ds, uint32_t len,
+                                           Acc& a) {
+    uint32_t sf = a.sf, c = 0, lk = 0, uk = 0;
     for (uint32_t i = 0; i < len; i++) {
         const uint32_t z = y << 2;
-        asm("{\n\t.reg .pred pl, ps, pc;\n\t.reg .b32 b, k;\n\t"
-            "setp.lt.u32 pl, %4, %6;\n\t"
-            "setp.lt.u32 ps, %5, %7;\n\t"
-            "@ps add.u32 %0, %0, 1;\n\t"
-            "vote.sync.ballot.b32 b, pl, 0xffffffff;\n\t"
-            "popc.b32 k, b;\n\t"
-            "add.u32 %2, %2, k;\n\t"
-            "setp.le.u32 pc, k, %8;\n\t"
-            "@pc add.u32 %1, %1, 1;\n\t"
-            "@!pc add.u32 %3, %3, k;\n\t}"
-            : "+r"(sf), "+r"(c), "+r"(lk), "+r"(uk)
-            : "r"(y), "r"(z), "r"(dl), "r"(ds), "r"(tm1));
+        const uint32_t k = __popc(__ballot_sync(kFull, y < dl));
+        sf += z < ds;
+        lk += k;
+        const bool coal = k <= 3;
+        c += coal;
+        uk += coal ? 0 : k;
         y += step;
     }
     a.sf = sf;
-    a.C2 = c;
-    a.lk = lk;
-    a.uk = uk;
-    a.W2 += len;
+    a.C += c;
+    a.lk += lk;
+    a.uk += uk;
+    a.W += len;
 }
 
 // MATCH: literal __match_any_sync expansion over 64-bit lane addresses.
@@ -165,17 +211,17 @@ __device__ __forceinline__ void hot_match(int64_t addr, int64_t step, uint32_t l
         const uint32_t lines = __popc(__ballot_sync(kFull, (ml & lt) == 0));
         const uint32_t sectors = __popc(__ballot_sync(kFull, (ms & lt) == 0));
         const bool coal = lines <= tmin;
-        L += lines;
-        S += sectors;
+        L += lines - 1;
+        S += sectors - 1;
         C += coal;
-        U += coal ? 0 : lines;
+        U += coal ? 0 : lines - 1;
         addr += step;
     }
-    a.lk += L;      // MATCH: lk = lines, uk = uncoalesced lines, sf(lane 0) = sectors
+    a.lk += L;
+    a.sk += S;
     a.uk += U;
-    a.sf += S;
-    a.C1 += C;
-    a.W1 += len;
+    a.C += C;
+    a.W += len;
 }
 
 // --------------------------------------------------------- warp iterator
@@ -229,7 +275,7 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
 // ------------------------------------------------------------- per access
 // Count WAs [off, off + cnt) of access `a` (instance order: warp-rep, then
 // inner tuple with the last inner loop fastest).  DEPTH = a.depth.
-template <bool MATCH, int DEPTH, bool T1>
+template <bool MATCH, int DEPTH, int TC>
 __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B, uint64_t T0,
                              uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t cnt, int lane, Acc& acc) {
     const uint32_t tmin = (32u * a.elem_bytes + 127u) / 128u;       // R11
@@ -284,8 +330,8 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
             } else {
                 const uint32_t y = (u_low + uint32_t(uint64_t(D))) << 25;
                 const uint32_t step = uint32_t(uint64_t(cl)) << 25;
-                if (T1) hot_t1(y, step, dl, ds, len, acc);
-                else hot_t2(y, step, dl, ds, len, tmin - 1, acc);
+                if (TC == 4) hot_row_t4(y, step, dl, ds, len, acc);
+                else hot_row<TC>(y, step, dl, ds, len, acc);
             }
             left -= len;
             // odometer carry (registers only)
@@ -302,26 +348,18 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     }
 }
 
-template <bool MATCH>
 __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
-    const uint32_t W = acc.W1 + acc.W2;
-    uint64_t L, S, C, U;
-    if (MATCH) {
-        L = acc.lk;
-        S = acc.sf;
-        C = acc.C1;
-        U = acc.uk;
-    } else {
-        const uint64_t slf = __reduce_add_sync(kFull, acc.lf);
-        const uint64_t ssf = __reduce_add_sync(kFull, acc.sf);
-        L = uint64_t(W) + slf + acc.lk;
-        S = uint64_t(W) + ssf;
-        C = uint64_t(acc.C1) + acc.C2;
-        U = uint64_t(acc.W1 - acc.C1) + slf + uint64_t(acc.W2 - acc.C2) + acc.uk;
-    }
+    const uint64_t slf = __reduce_add_sync(kFull, acc.lf);
+    const uint64_t ssf = __reduce_add_sync(kFull, acc.sf);
+    const uint64_t suf = __reduce_add_sync(kFull, acc.uf);
+    const uint64_t W = acc.W;
+    const uint64_t L = W + slf + acc.lk;
+    const uint64_t S = W + ssf + acc.sk;
+    const uint64_t C = acc.C;
+    const uint64_t U = (W - C) + suf + acc.uk;
     if (W && lane < 5) {
         const uint64_t v = lane == 0 ? W : lane == 1 ? L : lane == 2 ? S : lane == 3 ? C : U;
-        atomicAdd(&a.prob_cnt[q * 5 + lane], (unsigned long long)v);
+        atomicAdd(&a.prob_cnt[q * kCntStride + lane], (unsigned long long)v);
     }
     acc = Acc{};
 }
@@ -344,37 +382,35 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
             continue;
         }
         const uint32_t t = uint32_t(umin64(Wk - off, take));
-        const bool t1 = ac.elem_bytes <= 4;                     // tmin = ceil(32 e / 128) = 1
+        const int tc = (32 * int(ac.elem_bytes) + 127) / 128;     // tmin (R11): 1, 2 or 4
+#define SEL_DISPATCH(M, TCV)                                                                          \
+    switch (d) {                                                                                      \
+    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
+    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
+    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
+    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;       \
+    }
         if (MATCH) {
-            switch (d) {
-            case 0: count_access<true, 0, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 1: count_access<true, 1, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 2: count_access<true, 2, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            default: count_access<true, 3, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            }
-        } else if (t1) {
-            switch (d) {
-            case 0: count_access<false, 0, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 1: count_access<false, 1, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 2: count_access<false, 2, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            default: count_access<false, 3, true>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            }
+            SEL_DISPATCH(true, 1)
+        } else if (tc == 1) {
+            SEL_DISPATCH(false, 1)
+        } else if (tc == 2) {
+            SEL_DISPATCH(false, 2)
         } else {
-            switch (d) {
-            case 0: count_access<false, 0, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 1: count_access<false, 1, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            case 2: count_access<false, 2, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            default: count_access<false, 3, false>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;
-            }
+            SEL_DISPATCH(false, 4)
         }
+#undef SEL_DISPATCH
         take -= t;
         off = 0;
     }
-    flush<MATCH>(a, q, acc, lane);
+    flush(a, q, acc, lane);
 }
 
 template <bool MATCH>
-__global__ void __launch_bounds__(256, 3) k_count(CountArgs a) {
+#ifndef SEL_COUNT_MIN_BLOCKS
+#define SEL_COUNT_MIN_BLOCKS 3
+#endif
+__global__ void __launch_bounds__(256, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;

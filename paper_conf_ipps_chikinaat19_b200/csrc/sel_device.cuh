@@ -14,6 +14,7 @@ constexpr uint64_t kLim48 = 1ull << 48;
 constexpr uint64_t kLim40 = 1ull << 40;
 constexpr uint32_t kNoProblem = 0xffffffffu;
 constexpr int kSlots = 8;              // distinct B classes shared per nest before overflow
+constexpr int kCntStride = 6;          // per problem: W, L, S, C, U (atomic), M_it (closed form)
 
 // ------------------------------------------------------------------ workspace
 // All offsets are 256-byte aligned.  Sized for the worst case of one counting
@@ -53,7 +54,7 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
     L.prob_B = o;     o = ws_align(o + n * sizeof(uint32_t));
     L.prob_W = o;     o = ws_align(o + (n + 1) * sizeof(uint64_t));
     L.prob_WR = o;    o = ws_align(o + n * sizeof(uint64_t));
-    L.prob_cnt = o;   o = ws_align(o + n * 5 * sizeof(uint64_t));
+    L.prob_cnt = o;   o = ws_align(o + n * kCntStride * sizeof(uint64_t));
     L.prob_status = o; o = ws_align(o + n);
     L.cand_status = o; o = ws_align(o + n);
     uint64_t big = n > n_nests ? n : n_nests;

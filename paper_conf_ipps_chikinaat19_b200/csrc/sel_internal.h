@@ -52,4 +52,8 @@ cudaError_t launch_model_from_counts(const sel_candidate* cands, uint64_t n, con
 cudaError_t launch_select(const sel_candidate* cands, uint64_t n, const double* t_gpu, const uint8_t* status,
                           uint8_t* decision, cudaStream_t s);
 
+// sel_next.cu (NEXT rows)
+cudaError_t launch_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
+                                 uint64_t n_groups, uint32_t* best, double* best_t, cudaStream_t s);
+
 }  // namespace sel

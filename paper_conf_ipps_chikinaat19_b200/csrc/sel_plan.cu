@@ -222,7 +222,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader*
     const uint64_t nq = hdr->n_problems;
     const uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (q >= nq) return;
-    for (int f = 0; f < 5; f++) prob_cnt[q * 5 + f] = 0;
+    for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
     const uint32_t nid = prob_nest[q];
     if (nid == kNoProblem) { prob_W[q] = 0; prob_WR[q] = 0; prob_status[q] = SEL_EINVAL; return; }
     const sel_nest nest = t.nests[nid];
@@ -232,6 +232,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader*
     if (st) { prob_W[q] = 0; prob_WR[q] = 0; return; }
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
+    prob_cnt[q * kCntStride + 5] = M_it;
     prob_W[q] = WR * M_it;
 }
 

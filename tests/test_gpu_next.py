@@ -1,0 +1,47 @@
+"""GPU parity of the NEXT rows against the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def sel():
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_chikinaat19_b200 as s
+    return s
+
+
+def test_select_launch_random(sel):
+    rng = np.random.default_rng(11)
+    n, G = 200000, 30000
+    group = rng.integers(0, G + 50, n).astype(np.uint32)
+    t = rng.choice([0.25, 1.0, 3.0, np.inf], n) * rng.integers(1, 5, n)
+    st = (rng.random(n) < 0.05).astype(np.uint8)
+    b_ref, v_ref = oracle.select_launch(group, t, st, G)
+    g_d = torch.from_numpy(group.view(np.int32)).cuda()
+    best, val = sel.select_launch(g_d, torch.from_numpy(t).cuda(), torch.from_numpy(st).cuda(), G)
+    torch.cuda.synchronize()
+    assert (best.cpu().numpy().view(np.uint32) == b_ref).all()
+    v = val.cpu().numpy()
+    assert ((v == v_ref) | (np.isinf(v) & np.isinf(v_ref))).all()
+
+
+def test_select_launch_on_c4(sel):
+    """c4: each of the 24 nests under 8 launch configurations -> the launch
+    with the lowest predicted T_gpu per nest, from the fused evaluation."""
+    b = gen.generate(4)
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
+    c = sel._as_bytes_tensor(b.cands, "candidate")
+    r = ev.evaluate(c, want_t_gpu=True)
+    group = torch.from_numpy(b.cands["nest_id"].astype(np.int32)).cuda()
+    best, val = sel.select_launch(group, r["t_gpu"], r["status"], 24)
+    torch.cuda.synchronize()
+    b_ref, v_ref = oracle.select_launch(b.cands["nest_id"], r["t_gpu"].cpu().numpy(), r["status"].cpu().numpy(), 24)
+    assert (best.cpu().numpy().view(np.uint32) == b_ref).all()
+    assert (val.cpu().numpy() == v_ref).all()

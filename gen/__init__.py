@@ -45,6 +45,12 @@ COUNTS_DTYPE = np.dtype([
     ("coalesced", "<u8"), ("uncoal_lines", "<u8"), ("warp_reps", "<u8"),
 ])
 
+CPU_PARAMS_DTYPE = np.dtype([
+    ("cpu_hz", "<f8"), ("tlb_entries", "<f8"), ("tlb_miss_cycles", "<f8"), ("loop_overhead_cycles", "<f8"),
+    ("schedule_static_cycles", "<f8"), ("sync_cycles", "<f8"), ("startup_cycles", "<f8"), ("page_bytes", "<f8"),
+])
+CPU_INPUT_DTYPE = np.dtype([("mca_cycles_per_iter", "<f8"), ("threads", "<u4"), ("_pad", "<u4")])
+
 TRIP_UNKNOWN = 0xFFFFFFFF  # unknown trip counts are assumed to be 128
 DEVICE_NAMES = ("K80", "P100", "V100", "B200")
 V100 = 2
@@ -77,6 +83,8 @@ def lib():
         L.selgen_shape_name.argtypes = [ctypes.c_int]
         L.selgen_count_indices.argtypes = [ctypes.c_int, vp, u64, ctypes.POINTER(u64)]
         L.selgen_fill_indices.argtypes = [ctypes.c_int, vp, u64, vp, vp, vp]
+        L.selgen_cpu_inputs.argtypes = [ctypes.c_int, u64, u64, vp]
+        L.selgen_cpu_params.argtypes = [vp]
         L.selgen_rng.restype = u64
         L.selgen_rng.argtypes = [u64, u64]
         _lib = L
@@ -157,6 +165,23 @@ def generate_indices(cfg: int, idx) -> Batch:
                              acc.ctypes.data) != 0:
         raise ValueError("selgen_fill_indices failed")
     return Batch(cands, nests, acc, launches(cfg), device_sets())
+
+
+def cpu_inputs(cfg: int, c0: int = 0, c1: int | None = None) -> np.ndarray:
+    """NEXT row f1 inputs (MCA stand-in cycles per parallel iteration, threads)."""
+    if c1 is None:
+        c1 = num_candidates(cfg)
+    out = np.zeros(c1 - c0, CPU_INPUT_DTYPE)
+    if lib().selgen_cpu_inputs(cfg, c0, c1, out.ctypes.data) != 0:
+        raise ValueError("bad range")
+    return out
+
+
+def cpu_params() -> np.ndarray:
+    """Table II constants + page size, one record."""
+    out = np.zeros(1, CPU_PARAMS_DTYPE)
+    lib().selgen_cpu_params(out.ctypes.data)
+    return out
 
 
 def rng(seed: int, i: int) -> int:

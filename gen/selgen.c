@@ -472,3 +472,55 @@ int selgen_fill_indices(int cfg, const uint64_t* idx, uint64_t m, gen_candidate*
     }
     return 0;
 }
+
+/* ------------------------------------------------------------ CPU inputs */
+/* Inputs of the NEXT-row f1 CPU model (Liao-Chapman, Fig. 3): the LLVM-MCA
+ * stand-in cycles per parallel iteration (mca_k x product of inner trips,
+ * the same synthetic loadout that produced cpu_cycles above) and the host
+ * thread count.  With a TLB term of zero the modelled cost equals the
+ * supplied cpu_cycles of the candidate. */
+static void cand_cpu(int cfg, uint64_t c, double* mca, uint32_t* threads) {
+    nest_params np;
+    const shape* sh;
+    int col = 0;
+    if (cfg == SELGEN_C3) {
+        *mca = 2.5;
+        *threads = ((c >> 1) & 1) ? 4u : 160u;
+        return;
+    }
+    if (cfg == SELGEN_C1) { sh = &SHAPES[0]; col = (int)c; shape_params(sh, cfg, 0, col, &np); }
+    else if (cfg == SELGEN_C2) {
+        int idx = (int)(c / 4), s = c2_nest(idx, &col);
+        sh = &SHAPES[s];
+        shape_params(sh, cfg, 0, col, &np);
+        np.threads = (idx & 1) ? 4 : 160;
+    } else if (cfg == SELGEN_C4) { sh = &SHAPES[c / 8]; shape_params(sh, cfg, 0, 0, &np); }
+    else { uint64_t g = c / 32; sh = &SHAPES[g % 24]; shape_params(sh, cfg, g / 24, 0, &np); }
+    uint64_t inner = 1;
+    for (int j = 0; j < sh->n_inner - (col ? 1 : 0); j++) inner *= col ? np.ext[2] : np.ext[1 + j];
+    *mca = (2.0 + 0.5 * (double)sh->n_acc) * (double)inner;
+    *threads = (uint32_t)np.threads;
+}
+
+int selgen_cpu_inputs(int cfg, uint64_t c0, uint64_t c1, gen_cpu_input* out) {
+    if (c0 > c1 || c1 > selgen_num_candidates(cfg)) return -1;
+    for (uint64_t c = c0; c < c1; c++) {
+        out[c - c0].mca_cycles_per_iter = 0.0;
+        out[c - c0]._pad = 0;
+        cand_cpu(cfg, c, &out[c - c0].mca_cycles_per_iter, &out[c - c0].threads);
+    }
+    return 0;
+}
+
+void selgen_cpu_params(gen_cpu_params* p) {
+    /* Table II plus the 64 KiB base page of Linux on POWER9
+     * (the page size is not in the paper; reading F1c). */
+    p->cpu_hz = 3.0e9;
+    p->tlb_entries = 1024.0;
+    p->tlb_miss_cycles = 14.0;
+    p->loop_overhead_cycles = 4.0;
+    p->schedule_static_cycles = 10154.0;
+    p->sync_cycles = 4000.0;
+    p->startup_cycles = 3000.0;
+    p->page_bytes = 65536.0;
+}

@@ -54,6 +54,18 @@ typedef struct {                       /* 24 bytes */
     double cpu_cycles, cpu_hz;
 } gen_candidate;
 
+/* NEXT row f1 (Liao-Chapman CPU model) inputs: Table II constants and the
+ * per-candidate LLVM-MCA stand-in cost per parallel iteration + threads. */
+typedef struct {                       /* 64 bytes */
+    double cpu_hz, tlb_entries, tlb_miss_cycles, loop_overhead_cycles,
+           schedule_static_cycles, sync_cycles, startup_cycles, page_bytes;
+} gen_cpu_params;
+
+typedef struct {                       /* 16 bytes */
+    double mca_cycles_per_iter;
+    uint32_t threads, _pad;
+} gen_cpu_input;
+
 /* Config ids follow BASELINE.json "configs" order, 1-based. */
 enum { SELGEN_C1 = 1, SELGEN_C2 = 2, SELGEN_C3 = 3, SELGEN_C4 = 4, SELGEN_C5 = 5 };
 
@@ -74,6 +86,9 @@ int selgen_fill(int cfg, uint64_t c0, uint64_t c1,
 int selgen_count_indices(int cfg, const uint64_t* idx, uint64_t m, uint64_t* n_access);
 int selgen_fill_indices(int cfg, const uint64_t* idx, uint64_t m, gen_candidate* cands, gen_nest* nests,
                         gen_access* acc);
+/* f1 inputs of candidates [c0, c1) and the Table II parameter set. */
+int selgen_cpu_inputs(int cfg, uint64_t c0, uint64_t c1, gen_cpu_input* out);
+void selgen_cpu_params(gen_cpu_params* p);
 /* Shape catalogue (24 Polybench-style sub-kernels). */
 int selgen_num_shapes(void);
 const char* selgen_shape_name(int s);

@@ -58,6 +58,7 @@ def lib():
                                       ctypes.c_int]
         L.oracle_model.argtypes = [vp, vp, vp, vp, vp, vp]
         L.oracle_select_launch.argtypes = [vp, u64, vp, vp, u64, vp, vp]
+        L.oracle_cpu_model.argtypes = [vp, vp, u64, vp, vp, u64, vp, vp]
         L.oracle_sizeof.restype = ctypes.c_size_t
         L.oracle_sizeof.argtypes = [ctypes.c_int]
         L.oracle_offsetof.restype = ctypes.c_size_t
@@ -117,6 +118,20 @@ def select_launch(group_of, t_gpu, status, n_groups):
     lib().oracle_select_launch(g.ctypes.data, len(g), t.ctypes.data, s.ctypes.data, n_groups, best.ctypes.data,
                                val.ctypes.data)
     return best, val
+
+
+def cpu_model(params, batch, cpu_in):
+    """NEXT row f1: (cpu_cycles f64[n], status u8[n]) -- Liao-Chapman Fig. 3 with Table II."""
+    n = len(batch.cands)
+    cyc = np.zeros(n, np.float64)
+    st = np.zeros(n, np.uint8)
+    p = np.ascontiguousarray(params)
+    ne = np.ascontiguousarray(batch.nests)
+    c = np.ascontiguousarray(batch.cands)
+    ci = np.ascontiguousarray(cpu_in)
+    lib().oracle_cpu_model(p.ctypes.data, ne.ctypes.data, len(ne), c.ctypes.data, ci.ctypes.data, n,
+                           cyc.ctypes.data, st.ctypes.data)
+    return cyc, st
 
 
 def layout(which: int):

@@ -426,3 +426,46 @@ void oracle_select_launch(const uint32_t* group_of, uint64_t n, const double* t_
         if (best[g] == 0xFFFFFFFFu || t_gpu[c] < best_val[g]) { best[g] = (uint32_t)c; best_val[g] = t_gpu[c]; }
     }
 }
+
+/* -------------------------------------------------- NEXT row f1 (CPU) */
+/* Liao-Chapman OpenMP cost model (Fig. 3) with the Table II
+ * parameters, for a target region holding one statically
+ * scheduled parallel for (the paper's kernels are "strictly parallel loop
+ * code").  Written out in the order of Fig. 3:
+ *   Chunk_size     = ceil(P / threads)               static schedule (F1a)
+ *   Cache_c        = TLB misses x TLB miss penalty   (F1c: misses = pages of
+ *                    the thread's share of the data beyond the TLB entries)
+ *   Loop_chunk_c   = Machine_c x per_iter x Chunk_size + Cache_c + Loop_overhead_c
+ *                    with Loop_overhead_c = Loop_overhead_per_iter x Chunk_size
+ *   Parallel_for_c = Schedule_times x (Schedule_c + Loop_chunk_c + Ordered_c + Reduction_c)
+ *                    Schedule_times = 1, Ordered = Reduction = 0        (F1b)
+ *   Thread_exe     = Parallel_for_c + Synchronization_c (implicit barrier)
+ *   Parallel_Region = Fork_c + max_threads(Thread_exe) + Join_c
+ *                    Fork = Par_Startup, Join folded into the barrier    (F1d)
+ * Machine_c x per_iter is the LLVM-MCA cost of one parallel iteration
+ * (P:L107-109), an input.  Status: EINVAL for a bad nest id, threads = 0 or a
+ * negative / non-finite MCA cost. */
+void oracle_cpu_model(const or_cpu_params* p, const or_nest* nests, uint64_t n_nests, const or_candidate* cands,
+                      const or_cpu_input* in, uint64_t n, double* cpu_cycles, uint8_t* status) {
+    for (uint64_t c = 0; c < n; c++) {
+        cpu_cycles[c] = 0.0;
+        status[c] = OR_OK;
+        const double mca = in[c].mca_cycles_per_iter;
+        if (cands[c].nest_id >= n_nests || in[c].threads == 0 || !(mca >= 0.0) || !isfinite(mca)) {
+            status[c] = OR_EINVAL;
+            continue;
+        }
+        const or_nest* nt = &nests[cands[c].nest_id];
+        const uint64_t P = nt->P0 * nt->P1;
+        const uint64_t chunk = ceil_div(P, in[c].threads);
+        const double footprint = (double)(nt->bytes_h2d + nt->bytes_d2h) / (double)in[c].threads;
+        const double pages = ceil(footprint / p->page_bytes);
+        const double misses = pages > p->tlb_entries ? pages - p->tlb_entries : 0.0;
+        const double cache = misses * p->tlb_miss_cycles;
+        const double loop_overhead = p->loop_overhead_cycles * (double)chunk;
+        const double loop_chunk = (mca * (double)chunk + cache) + loop_overhead;
+        const double parallel_for = 1.0 * (((p->schedule_static_cycles + loop_chunk) + 0.0) + 0.0);
+        const double thread_exe = parallel_for + p->sync_cycles;
+        cpu_cycles[c] = (p->startup_cycles + thread_exe) + 0.0;
+    }
+}

@@ -44,6 +44,13 @@ typedef struct {
     double cpu_cycles, cpu_hz;
 } or_candidate;
 
+/* NEXT row f1 inputs (same layouts as gen/selgen.h, declared independently) */
+typedef struct {
+    double cpu_hz, tlb_entries, tlb_miss_cycles, loop_overhead_cycles,
+           schedule_static_cycles, sync_cycles, startup_cycles, page_bytes;
+} or_cpu_params;
+typedef struct { double mca_cycles_per_iter; uint32_t threads, _pad; } or_cpu_input;
+
 /* Everything the oracle computes for one candidate: the hot path's outputs
  * (counts, cycles, t_gpu, decision, status) plus the model's intermediate
  * values, exposed so that tests can pin them against closed forms. */
@@ -86,6 +93,10 @@ void oracle_model(const or_device* dev, const or_nest* nest, const or_access* ac
  * +inf: lowest index; no valid candidate: best = 0xFFFFFFFF, +inf). */
 void oracle_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
                           uint64_t n_groups, uint32_t* best, double* best_val);
+
+/* NEXT row f1: Liao-Chapman CPU cycles (Fig. 3 + Table II) per candidate. */
+void oracle_cpu_model(const or_cpu_params* p, const or_nest* nests, uint64_t n_nests, const or_candidate* cands,
+                      const or_cpu_input* in, uint64_t n, double* cpu_cycles, uint8_t* status);
 
 /* Layout self-description for tests/test_layout.py. */
 size_t oracle_sizeof(int which);

@@ -171,6 +171,22 @@ def select_launch(group_of: torch.Tensor, t_gpu: torch.Tensor, status: torch.Ten
     return best, best_t
 
 
+def model_cpu_cost(cands: torch.Tensor, tables: DeviceTables, cpu_in, params, stream=None) -> torch.Tensor:
+    """sel_model_cpu_cost (NEXT row f1): overwrite the candidates' cpu_cycles /
+    cpu_hz with the Liao-Chapman model; returns status uint8[n]."""
+    _require_cuda(cands)
+    n = _n(cands, "candidate")
+    cin = cpu_in if isinstance(cpu_in, torch.Tensor) else torch.from_numpy(
+        np.ascontiguousarray(cpu_in).view(np.uint8).reshape(-1)).to(cands.device)
+    p = np.ascontiguousarray(params)
+    if p.dtype.itemsize != 64:
+        raise ValueError("CPU parameter record must be 64 bytes")
+    status = torch.empty(n, dtype=torch.uint8, device=cands.device)
+    _lib.check(_lib.lib().sel_model_cpu_cost(_ptr(cands), n, tables.ref(), _ptr(cin), p.ctypes.data,
+                                             _ptr(status), _stream(stream)))
+    return status
+
+
 def read_stats(workspace: torch.Tensor, stream=None) -> dict:
     st = _lib.Stats()
     wp, _ = _ws_ptr(workspace)
@@ -210,6 +226,7 @@ sel_select = select
 sel_evaluate = evaluate
 sel_read_stats = read_stats
 sel_select_launch = select_launch
+sel_model_cpu_cost = model_cpu_cost
 
 
 class Evaluator:

@@ -197,6 +197,19 @@ int sel_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu,
     return SEL_OK;
 }
 
+int sel_model_cpu_cost(sel_candidate* c, uint64_t n, const sel_tables* t, const sel_cpu_input* in,
+                       const sel_cpu_params* p, uint8_t* status, sel_stream_t stream) {
+    if (int r = check_tables(t)) return r;
+    if (n == 0) return SEL_OK;
+    if (!c || !in || !p || !status) return fail(SEL_EINVAL, "NULL argument%s");
+    if (!(p->cpu_hz > 0) || !(p->page_bytes > 0) || p->tlb_entries < 0 || p->tlb_miss_cycles < 0 ||
+        p->loop_overhead_cycles < 0 || p->schedule_static_cycles < 0 || p->sync_cycles < 0 || p->startup_cycles < 0)
+        return fail(SEL_EINVAL, "invalid CPU parameter set%s");
+    cudaError_t e = launch_cpu_model(c, n, *t, in, *p, status, reinterpret_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "model_cpu_cost");
+    return SEL_OK;
+}
+
 int sel_read_stats(const void* ws, sel_stats* out, sel_stream_t stream) {
     if (!ws || !out) return fail(SEL_EINVAL, "NULL argument%s");
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
@@ -292,3 +305,5 @@ static_assert(sizeof(sel_launch) == 16, "sel_launch layout");
 static_assert(sizeof(sel_candidate) == 24, "sel_candidate layout");
 static_assert(sizeof(sel_counts) == 48, "sel_counts layout");
 static_assert(sizeof(sel_stats) == 64, "sel_stats layout");
+static_assert(sizeof(sel_cpu_params) == 64, "sel_cpu_params layout");
+static_assert(sizeof(sel_cpu_input) == 16, "sel_cpu_input layout");

@@ -56,4 +56,7 @@ cudaError_t launch_select(const sel_candidate* cands, uint64_t n, const double* 
 cudaError_t launch_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
                                  uint64_t n_groups, uint32_t* best, double* best_t, cudaStream_t s);
 
+cudaError_t launch_cpu_model(sel_candidate* cands, uint64_t n, const sel_tables& t, const sel_cpu_input* in,
+                             const sel_cpu_params& p, uint8_t* status, cudaStream_t s);
+
 }  // namespace sel

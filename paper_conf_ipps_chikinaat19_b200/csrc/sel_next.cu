@@ -62,3 +62,49 @@ cudaError_t launch_select_launch(const uint32_t* group_of, uint64_t n, const dou
 }
 
 }  // namespace sel
+
+// f1  Liao-Chapman CPU cost model (Fig. 3; Table II)
+//     on the device, so the CPU side of the decision is modelled rather than
+//     supplied: one thread per candidate evaluates the Fig. 3 sequence for a
+//     statically scheduled parallel for and writes the result into the
+//     candidate's cpu_cycles / cpu_hz (readings F1a-F1d in DESIGN.md).
+//     fp64 with explicit round-to-nearest intrinsics, same order as the oracle.
+namespace sel {
+
+__global__ void __launch_bounds__(256) k_cpu_model(sel_candidate* __restrict__ cands, uint64_t n, sel_tables t,
+                                                   const sel_cpu_input* __restrict__ in, sel_cpu_params p,
+                                                   uint8_t* __restrict__ status) {
+    const uint64_t c = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (c >= n) return;
+    const sel_cpu_input x = in[c];
+    const uint32_t nid = cands[c].nest_id;
+    if (nid >= t.n_nests || x.threads == 0 || !(x.mca_cycles_per_iter >= 0.0) || !isfinite(x.mca_cycles_per_iter)) {
+        status[c] = SEL_EINVAL;
+        return;
+    }
+    const sel_nest nt = t.nests[nid];
+    const uint64_t P = nt.P0 * nt.P1;
+    const uint64_t chunk = cdiv(P, x.threads);                                     // F1a
+    const double footprint = __ddiv_rn(__ull2double_rn(nt.bytes_h2d + nt.bytes_d2h), __uint2double_rn(x.threads));
+    const double pages = ceil(__ddiv_rn(footprint, p.page_bytes));
+    const double misses = pages > p.tlb_entries ? __dsub_rn(pages, p.tlb_entries) : 0.0;
+    const double cache = __dmul_rn(misses, p.tlb_miss_cycles);                     // F1c
+    const double loop_overhead = __dmul_rn(p.loop_overhead_cycles, __ull2double_rn(chunk));
+    const double loop_chunk = __dadd_rn(__dadd_rn(__dmul_rn(x.mca_cycles_per_iter, __ull2double_rn(chunk)), cache),
+                                        loop_overhead);
+    const double parallel_for = __dmul_rn(1.0, __dadd_rn(__dadd_rn(__dadd_rn(p.schedule_static_cycles, loop_chunk), 0.0),
+                                                         0.0));                   // F1b
+    const double thread_exe = __dadd_rn(parallel_for, p.sync_cycles);
+    cands[c].cpu_cycles = __dadd_rn(__dadd_rn(p.startup_cycles, thread_exe), 0.0);  // F1d
+    cands[c].cpu_hz = p.cpu_hz;
+    status[c] = SEL_OK;
+}
+
+cudaError_t launch_cpu_model(sel_candidate* cands, uint64_t n, const sel_tables& t, const sel_cpu_input* in,
+                             const sel_cpu_params& p, uint8_t* status, cudaStream_t s) {
+    k_cpu_model<<<unsigned((n + 255) / 256), 256, 0, s>>>(cands, n, t, in, p, status);
+    note_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace sel

@@ -45,3 +45,30 @@ def test_select_launch_on_c4(sel):
     b_ref, v_ref = oracle.select_launch(b.cands["nest_id"], r["t_gpu"].cpu().numpy(), r["status"].cpu().numpy(), 24)
     assert (best.cpu().numpy().view(np.uint32) == b_ref).all()
     assert (val.cpu().numpy() == v_ref).all()
+
+
+@pytest.mark.parametrize("cfg,rng", [(1, (0, 2)), (2, (0, 108)), (4, (0, 192)), (5, (0, 2000000))])
+def test_cpu_model_parity(sel, cfg, rng):
+    """NEXT row f1: the device Liao-Chapman model writes the same cpu_cycles
+    (bit-exact) and statuses as the oracle; c4 exercises the TLB term."""
+    b = gen.generate(cfg, *rng)
+    cin = gen.cpu_inputs(cfg, *rng)
+    cin["threads"][::97] = 0                                  # some invalid inputs
+    ref, st_ref = oracle.cpu_model(gen.cpu_params(), b, cin)
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
+    c = sel._as_bytes_tensor(b.cands.copy(), "candidate")
+    st = sel.model_cpu_cost(c, ev.tables, cin, gen.cpu_params())
+    torch.cuda.synchronize()
+    out = c.cpu().numpy().view(gen.CANDIDATE_DTYPE)
+    st = st.cpu().numpy()
+    assert (st == st_ref).all()
+    ok = st == 0
+    assert (out["cpu_cycles"][ok] == ref[ok]).all()
+    assert (out["cpu_hz"][ok] == 3e9).all()
+    assert (out["cpu_cycles"][~ok] == b.cands["cpu_cycles"][~ok]).all()    # invalid: untouched
+    # the modelled cost then drives the decision exactly like a supplied one
+    if cfg in (1, 2):
+        r = ev.evaluate(c, want_t_gpu=True)
+        bb = gen.Batch(out.copy(), b.nests, b.accesses, b.launches, b.devices)
+        ref_eval = oracle.evaluate(bb)
+        assert (r["decision"].cpu().numpy() == ref_eval["decision"]).all()

@@ -20,3 +20,68 @@ def test_select_launch_matches_numpy_argmin():
         m = t[idx].min()
         first = idx[np.nonzero(t[idx] == m)[0][0]]                # ties: lowest index
         assert best[g] == first and val[g] == m
+
+
+# ---------------------------------------------------------------- f1 (CPU model)
+import gen  # noqa: E402
+
+
+def _one_nest(P, bytes_total=0):
+    n = np.zeros(1, gen.NEST_DTYPE)
+    n["P0"], n["P1"], n["par_dims"] = P, 1, 1
+    n["bytes_h2d"] = bytes_total
+    c = np.zeros(1, gen.CANDIDATE_DTYPE)
+    return gen.Batch(c, n, np.zeros(1, gen.ACCESS_DTYPE), gen.launches(1), gen.device_sets())
+
+
+def _cin(mca, threads):
+    x = np.zeros(1, gen.CPU_INPUT_DTYPE)
+    x["mca_cycles_per_iter"], x["threads"] = mca, threads
+    return x
+
+
+def test_cpu_model_hand_values():
+    """Fig. 3 with Table II: Par_Startup 3000 + static schedule
+    10154 + Chunk x (Machine x per_iter + loop overhead 4) + sync 4000."""
+    p = gen.cpu_params()
+    cyc, st = oracle.cpu_model(p, _one_nest(1000), _cin(10.0, 160))
+    assert st[0] == 0 and cyc[0] == 3000 + 10154 + 7 * (10 + 4) + 4000
+    cyc, _ = oracle.cpu_model(p, _one_nest(1000), _cin(10.0, 1))            # one thread: chunk = P
+    assert cyc[0] == 17154 + 1000 * 14
+    cyc, _ = oracle.cpu_model(p, _one_nest(50), _cin(10.0, 160))            # more threads than iterations
+    assert cyc[0] == 17154 + 1 * 14
+
+
+def test_cpu_model_tlb_term():
+    """TLB term (F1c): misses = pages of the thread's share beyond the 1024
+    entries, 14 cycles each (Table II)."""
+    p = gen.cpu_params()
+    page = 65536
+    for extra in (0, 1, 10, 1000):
+        cyc, _ = oracle.cpu_model(p, _one_nest(160, (1024 + extra) * page * 4), _cin(1.0, 4))
+        assert cyc[0] == 17154 + 40 * (1 + 4) + 14 * extra
+    cyc, _ = oracle.cpu_model(p, _one_nest(160, 1024 * page * 4 - 1), _cin(1.0, 4))
+    assert cyc[0] == 17154 + 40 * 5
+
+
+def test_cpu_model_matches_supplied_synthetic_cost():
+    """Without TLB misses the modelled cost equals the synthetic cost the
+    generator supplies (same Fig. 3 form, written independently in gen/)."""
+    p = gen.cpu_params()
+    for cfg, rng in ((1, (0, 2)), (2, (0, 108)), (3, (0, 20000)), (5, (1234567, 1334567))):
+        b = gen.generate(cfg, *rng)
+        cyc, st = oracle.cpu_model(p, b, gen.cpu_inputs(cfg, *rng))
+        assert (st == 0).all()
+        np.testing.assert_array_equal(cyc, b.cands["cpu_cycles"])
+
+
+def test_cpu_model_monotone_and_invalid():
+    p = gen.cpu_params()
+    prev = 0
+    for mca in (0.0, 0.5, 1.0, 7.0, 100.0):
+        cyc, _ = oracle.cpu_model(p, _one_nest(777), _cin(mca, 8))
+        assert cyc[0] > prev
+        prev = cyc[0]
+    for bad in (_cin(1.0, 0), _cin(-1.0, 4), _cin(float("nan"), 4), _cin(float("inf"), 4)):
+        _, st = oracle.cpu_model(p, _one_nest(10), bad)
+        assert st[0] == oracle.EINVAL

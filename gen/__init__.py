@@ -30,7 +30,7 @@ ACCESS_DTYPE = np.dtype([
 ])
 NEST_DTYPE = np.dtype([
     ("P0", "<u8"), ("P1", "<u8"), ("trip", "<u4", (3,)), ("par_dims", "u1"), ("depth", "u1"),
-    ("_pad", "u1", (2,)), ("comp_insts", "<f8", (4,)), ("bytes_h2d", "<u8"), ("bytes_d2h", "<u8"),
+    ("n_sync", "<u2"), ("comp_insts", "<f8", (4,)), ("bytes_h2d", "<u8"), ("bytes_d2h", "<u8"),
     ("access_off", "<u4"), ("n_access", "<u4"),
 ])
 LAUNCH_DTYPE = np.dtype([

@@ -194,6 +194,14 @@ void oracle_model(const or_device* dev, const or_nest* nest, const or_access* ac
         }
         r->E = E;
         Exec = (E * Rep) * (double)r->R;                          /* x #Rep x #OMP_Rep */
+        if (nest->n_sync > 0) {
+            /* NEXT row f4, [H&K] synchronisation cost (readings F4a, F4b):
+             * Departure_delay x (MWP - 1) x #synch x #Active_blocks_per_SM
+             * x #Rep, once per OpenMP repetition. */
+            const double Sync = ((((r->Dep * (r->MWP - 1.0)) * (double)nest->n_sync) * (double)abps) * Rep)
+                                * (double)r->R;
+            Exec = Exec + Sync;
+        }
     }
     r->cycles = Exec;
     /* a7 (R20, R21) */
@@ -392,7 +400,7 @@ size_t oracle_offsetof(int which, int field) {
     static const size_t acc[] = {OFF(or_access, base), OFF(or_access, c_par), OFF(or_access, c_inner),
         OFF(or_access, elem_bytes), OFF(or_access, depth), OFF(or_access, is_store)};
     static const size_t nest[] = {OFF(or_nest, P0), OFF(or_nest, P1), OFF(or_nest, trip), OFF(or_nest, par_dims),
-        OFF(or_nest, depth), OFF(or_nest, comp_insts), OFF(or_nest, bytes_h2d), OFF(or_nest, bytes_d2h),
+        OFF(or_nest, depth), OFF(or_nest, n_sync), OFF(or_nest, comp_insts), OFF(or_nest, bytes_h2d), OFF(or_nest, bytes_d2h),
         OFF(or_nest, access_off), OFF(or_nest, n_access)};
     static const size_t lau[] = {OFF(or_launch, block), OFF(or_launch, grid_max), OFF(or_launch, regs_per_thread),
         OFF(or_launch, smem_per_block)};

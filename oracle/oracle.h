@@ -30,7 +30,8 @@ typedef struct {
 typedef struct {
     uint64_t P0, P1;
     uint32_t trip[3];
-    uint8_t par_dims, depth, _pad[2];
+    uint8_t par_dims, depth;
+    uint16_t n_sync;
     double comp_insts[4];
     uint64_t bytes_h2d, bytes_d2h;
     uint32_t access_off, n_access;

@@ -44,7 +44,7 @@ class Access(ctypes.Structure):
 
 class Nest(ctypes.Structure):
     _fields_ = [("P0", ctypes.c_uint64), ("P1", ctypes.c_uint64), ("trip", ctypes.c_uint32 * 3),
-                ("par_dims", ctypes.c_uint8), ("depth", ctypes.c_uint8), ("_pad", ctypes.c_uint8 * 2),
+                ("par_dims", ctypes.c_uint8), ("depth", ctypes.c_uint8), ("n_sync", ctypes.c_uint16),
                 ("comp_insts", ctypes.c_double * 4), ("bytes_h2d", ctypes.c_uint64),
                 ("bytes_d2h", ctypes.c_uint64), ("access_off", ctypes.c_uint32), ("n_access", ctypes.c_uint32)]
 

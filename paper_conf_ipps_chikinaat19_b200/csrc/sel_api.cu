@@ -274,7 +274,7 @@ size_t sel_offsetof(int which, int field) {
     static const size_t acc[] = {OFF(sel_access, base), OFF(sel_access, c_par), OFF(sel_access, c_inner),
         OFF(sel_access, elem_bytes), OFF(sel_access, depth), OFF(sel_access, is_store)};
     static const size_t nest[] = {OFF(sel_nest, P0), OFF(sel_nest, P1), OFF(sel_nest, trip), OFF(sel_nest, par_dims),
-        OFF(sel_nest, depth), OFF(sel_nest, comp_insts), OFF(sel_nest, bytes_h2d), OFF(sel_nest, bytes_d2h),
+        OFF(sel_nest, depth), OFF(sel_nest, n_sync), OFF(sel_nest, comp_insts), OFF(sel_nest, bytes_h2d), OFF(sel_nest, bytes_d2h),
         OFF(sel_nest, access_off), OFF(sel_nest, n_access)};
     static const size_t lau[] = {OFF(sel_launch, block), OFF(sel_launch, grid_max), OFF(sel_launch, regs_per_thread),
         OFF(sel_launch, smem_per_block)};

@@ -72,3 +72,13 @@ def test_cpu_model_parity(sel, cfg, rng):
         bb = gen.Batch(out.copy(), b.nests, b.accesses, b.launches, b.devices)
         ref_eval = oracle.evaluate(bb)
         assert (r["decision"].cpu().numpy() == ref_eval["decision"]).all()
+
+
+def test_sync_term_parity(sel):
+    """NEXT row f4: nests with barriers (n_sync > 0) -> bit-exact cycles."""
+    import test_gpu_parity as P
+    b = P._random_batch(5, 2000)
+    nests = b.nests.copy()
+    nests["n_sync"] = np.arange(len(nests)) % 4
+    bb = gen.Batch(b.cands, nests, b.accesses, b.launches, b.devices)
+    P.assert_parity(P.run_gpu(sel, bb), oracle.evaluate(bb), ctx="f4 sync")

@@ -85,3 +85,33 @@ def test_cpu_model_monotone_and_invalid():
     for bad in (_cin(1.0, 0), _cin(-1.0, 4), _cin(float("nan"), 4), _cin(float("inf"), 4)):
         _, st = oracle.cpu_model(p, _one_nest(10), bad)
         assert st[0] == oracle.EINVAL
+
+
+# ---------------------------------------------------------------- f4 (H&K synchronisation)
+def _with_sync(b, k):
+    n = b.nests.copy()
+    n["n_sync"] = k
+    return gen.Batch(b.cands, n, b.accesses, b.launches, b.devices)
+
+
+def test_sync_term_linear_and_zero_cases():
+    """[H&K] synchronisation cost Departure_delay x (MWP-1) x #synch x
+    #Active_blocks x #Rep (x #OMP_Rep, F4a): zero without barriers, linear in
+    the barrier count, zero when a single warp runs (MWP = 1)."""
+    b = gen.generate(2)
+    r0 = oracle.evaluate(b)
+    r1 = oracle.evaluate(_with_sync(b, 1))
+    r2 = oracle.evaluate(_with_sync(b, 2))
+    s1, s2 = r1["cycles"] - r0["cycles"], r2["cycles"] - r0["cycles"]
+    assert (s1 >= 0).all() and (s1 > 0).any()
+    np.testing.assert_allclose(s2, 2 * s1, rtol=1e-9)
+    m = r0["W"] > 0
+    expect = r0["Dep"] * (r0["MWP"] - 1.0) * r0["abps"].astype(float) * r0["Rep"] * r0["R"].astype(float)
+    np.testing.assert_allclose(s1[m], expect[m], rtol=1e-9)
+    np.testing.assert_array_equal(r1["hk_case"], r0["hk_case"])
+    # lone warp: MWP = N = 1 -> no synchronisation cost
+    a = gen.make_access(base=1 << 28, c_par=(4,), c_inner=(0,), elem_bytes=4, depth=1)
+    lau = np.zeros(1, gen.LAUNCH_DTYPE)
+    lau[0] = (32, 1, 0, 0)
+    one = gen.custom_batch([dict(P0=64, trip=[5], comp=[1.0, 2.0], accesses=[a])], launches_=lau)
+    assert oracle.evaluate(_with_sync(one, 3))["cycles"][0] == oracle.evaluate(one)["cycles"][0]

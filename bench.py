@@ -46,6 +46,7 @@ def parse():
     p.add_argument("--flags", type=int, default=0, help="libsel flags (1 no count sharing, 2 match_any)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-next", action="store_true", help="skip timing the NEXT rows f1-f3")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     return p.parse_args()
 
@@ -309,9 +310,76 @@ def run_ours(args):
             "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
             "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
+    if not args.no_next and args.config == 5:
+        line["next_rows"] = time_next_rows(sel, gen, ev, batch, cands, out, args, c0, c1, dev)
     if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_oracle_sample(batch, args.cpu_seconds, total)
     print(json.dumps(line), flush=True)
+
+
+def time_next_rows(sel, gen, ev, batch, cands, out, args, c0, c1, dev):
+    """NEXT rows on this rank's c5 batch: f2 symbolic IPDA
+    binding of every access, f1 Liao-Chapman CPU model of every candidate, f3
+    launch selection per (nest, device) group.  Device time with CUDA events
+    (best of 3 after a warm-up); results checked against the generator's
+    concrete accesses (f2) and the supplied CPU cost (f1, no TLB misses in c5)."""
+    import torch
+    import numpy as np
+
+    def timed(fn, reps=3):
+        fn()
+        torch.cuda.synchronize(dev)
+        best = 1e30
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            torch.cuda.synchronize(dev)
+            best = min(best, a.elapsed_time(b))
+        return best
+
+    res = {}
+    sym, terms = gen.sym_tables()
+    vals, items = gen.sym_instances(args.config, c0, c1)
+    sym_d, terms_d = sel._dev_bytes(sym, dev), sel._dev_bytes(terms, dev)
+    vals_d, items_d = sel._dev_bytes(vals, dev), sel._dev_bytes(items, dev)
+    bound = torch.empty(len(items) * 64, dtype=torch.uint8, device=dev)
+    st = torch.empty(len(items), dtype=torch.uint8, device=dev)
+    L = sel._lib.lib()
+
+    def f2():
+        sel._lib.check(L.sel_bind_accesses(sel._ptr(sym_d), len(sym), sel._ptr(terms_d), len(terms),
+                                           sel._ptr(vals_d), len(vals), sel._ptr(items_d), len(items),
+                                           sel._ptr(bound), sel._ptr(st), sel._stream()))
+    ms = timed(f2)
+    ok = bool(torch.equal(bound, ev.tables.accesses[: len(items) * 64])) and int(st.max().item()) == 0
+    nbytes = len(items) * (8 + 64 + 1) + 9 * 8 * len(batch.nests)
+    res["f2_bind"] = {"items": len(items), "ms": ms, "items_per_s": len(items) / (ms / 1e3),
+                      "hbm_gbs": nbytes / (ms / 1e3) / 1e9, "matches_generator": ok}
+
+    cin = sel._dev_bytes(gen.cpu_inputs(args.config, c0, c1), dev)
+    params = gen.cpu_params()
+    cc = cands.clone()
+
+    def f1():
+        sel.model_cpu_cost(cc, ev.tables, cin, params)
+    ms = timed(f1)
+    same = bool(torch.equal(cc, cands))
+    n = len(batch)
+    res["f1_cpu_model"] = {"candidates": n, "ms": ms, "candidates_per_s": n / (ms / 1e3),
+                           "hbm_gbs": n * (24 + 16 + 24 + 1) / (ms / 1e3) / 1e9, "equals_supplied_cost": same}
+
+    r = ev.evaluate(cands, want_t_gpu=True)
+    group = torch.from_numpy((batch.cands["nest_id"].astype(np.int64) * 4 + batch.cands["device_id"]).astype(
+        np.int32)).to(dev)
+    n_groups = len(batch.nests) * 4
+
+    def f3():
+        sel.select_launch(group, r["t_gpu"], r["status"], n_groups)
+    ms = timed(f3)
+    res["f3_select_launch"] = {"candidates": n, "groups": n_groups, "ms": ms, "candidates_per_s": n / (ms / 1e3)}
+    return res
 
 
 def main():

@@ -51,6 +51,12 @@ CPU_PARAMS_DTYPE = np.dtype([
 ])
 CPU_INPUT_DTYPE = np.dtype([("mca_cycles_per_iter", "<f8"), ("threads", "<u4"), ("_pad", "<u4")])
 
+SYM_TERM_DTYPE = np.dtype([("k", "<i8"), ("sym", "<u2", (3,)), ("_pad", "<u2")])
+SYM_ACCESS_DTYPE = np.dtype([("term_off", "<u4", (6,)), ("n_terms", "u1", (6,)), ("elem_sym", "<u2"),
+                             ("elem_bytes", "u1"), ("depth", "u1"), ("is_store", "u1"), ("_pad", "u1", (5,))])
+BIND_ITEM_DTYPE = np.dtype([("sym_access", "<u4"), ("frame", "<u4")])
+SYM_ONE = 0xFFFF
+
 TRIP_UNKNOWN = 0xFFFFFFFF  # unknown trip counts are assumed to be 128
 DEVICE_NAMES = ("K80", "P100", "V100", "B200")
 V100 = 2
@@ -85,6 +91,9 @@ def lib():
         L.selgen_fill_indices.argtypes = [ctypes.c_int, vp, u64, vp, vp, vp]
         L.selgen_cpu_inputs.argtypes = [ctypes.c_int, u64, u64, vp]
         L.selgen_cpu_params.argtypes = [vp]
+        L.selgen_sym_tables.argtypes = [vp, vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
+        L.selgen_sym_count.argtypes = [ctypes.c_int, u64, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
+        L.selgen_sym_fill.argtypes = [ctypes.c_int, u64, u64, vp, vp]
         L.selgen_rng.restype = u64
         L.selgen_rng.argtypes = [u64, u64]
         _lib = L
@@ -182,6 +191,33 @@ def cpu_params() -> np.ndarray:
     out = np.zeros(1, CPU_PARAMS_DTYPE)
     lib().selgen_cpu_params(out.ctypes.data)
     return out
+
+
+def sym_tables():
+    """NEXT row f2: (symbolic accesses, term pool) of the 24 shapes x {1-D, collapse}."""
+    L = lib()
+    ns, nt = ctypes.c_uint32(), ctypes.c_uint32()
+    L.selgen_sym_tables(None, None, ctypes.byref(ns), ctypes.byref(nt))
+    sym = np.zeros(ns.value, SYM_ACCESS_DTYPE)
+    terms = np.zeros(nt.value, SYM_TERM_DTYPE)
+    L.selgen_sym_tables(sym.ctypes.data, terms.ctypes.data, ctypes.byref(ns), ctypes.byref(nt))
+    return sym, terms
+
+
+def sym_instances(cfg: int, c0: int = 0, c1: int | None = None):
+    """NEXT row f2: (symbol frames int64, bind items) for the accesses that
+    ``generate(cfg, c0, c1)`` produces, in the same order (configs 2, 5)."""
+    L = lib()
+    if c1 is None:
+        c1 = num_candidates(cfg)
+    nv, ni = ctypes.c_uint64(), ctypes.c_uint64()
+    if L.selgen_sym_count(cfg, c0, c1, ctypes.byref(nv), ctypes.byref(ni)) != 0:
+        raise ValueError("symbolic instances exist for configs 2 and 5 only")
+    values = np.zeros(max(nv.value, 1), np.int64)
+    items = np.zeros(max(ni.value, 1), BIND_ITEM_DTYPE)
+    if L.selgen_sym_fill(cfg, c0, c1, values.ctypes.data, items.ctypes.data) != 0:
+        raise ValueError("selgen_sym_fill failed")
+    return values, items[:ni.value]
 
 
 def rng(seed: int, i: int) -> int:

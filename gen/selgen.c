@@ -524,3 +524,107 @@ void selgen_cpu_params(gen_cpu_params* p) {
     p->startup_cycles = 3000.0;
     p->page_bytes = 65536.0;
 }
+
+/* ------------------------------------------------------ symbolic accesses */
+/* NEXT row f2 inputs: the accesses of every shape as IPDA-style symbolic
+ * expressions: each byte coefficient is a sum of terms
+ * k * v[s0] * v[s1] * v[s2] over a per-nest-instance symbol frame
+ *   frame = [elem, size(sym0..sym3), array_offset(0..3)]           (9 values)
+ * Binding the frame reproduces exactly the concrete accesses selgen_fill
+ * writes.  Symbolic table index: (2 * shape + collapse) * 12 + access. */
+#define FR_ELEM 0
+#define FR_SIZE 1
+#define FR_OFF 5
+#define SYM_ONE 0xFFFFu
+
+static uint32_t sym_term(gen_sym_term* terms, uint32_t* nt, int64_t k, uint16_t s0, uint16_t s1, uint16_t s2) {
+    if (terms) { terms[*nt].k = k; terms[*nt].sym[0] = s0; terms[*nt].sym[1] = s1; terms[*nt].sym[2] = s2; terms[*nt]._pad = 0; }
+    return (*nt)++;
+}
+
+int selgen_sym_tables(gen_sym_access* sym, gen_sym_term* terms, uint32_t* n_sym, uint32_t* n_terms) {
+    uint32_t nt = 0;
+    for (int s = 0; s < 24; s++) {
+        const shape* sh = &SHAPES[s];
+        for (int col = 0; col < 2; col++) {
+            for (int k = 0; k < 12; k++) {
+                gen_sym_access* g = sym ? &sym[(2 * s + col) * 12 + k] : 0;
+                if (g) memset(g, 0, sizeof *g);
+                if (k >= sh->n_acc || (col && !sh->collapse_ok)) continue;
+                const sh_access* sa = &sh->acc[k];
+                const sh_array* ar = &sh->arr[sa->arr];
+                /* coefficient slots: 0 base, 1 c_par[0], 2 c_par[1], 3..5 c_inner[0..2] */
+                int slot_of_var[3];
+                if (col) { slot_of_var[0] = 1; slot_of_var[1] = 2; slot_of_var[2] = 3; }
+                else { slot_of_var[0] = 1; slot_of_var[1] = 3; slot_of_var[2] = 4; }
+                for (int slot = 0; slot < 6; slot++) {
+                    uint32_t first = nt, cnt = 0;
+                    if (slot == 0) {
+                        sym_term(terms, &nt, BASE0 + (int64_t)sa->arr * ARR_SPACING, SYM_ONE, SYM_ONE, SYM_ONE); cnt++;
+                        sym_term(terms, &nt, 1, (uint16_t)(FR_OFF + sa->arr), SYM_ONE, SYM_ONE); cnt++;
+                    }
+                    for (int d = 0; d < ar->ndims; d++) {
+                        int64_t kk = 0;
+                        if (slot == 0) kk = sa->idx[d][3];
+                        else for (int v = 0; v < 3; v++) if (slot_of_var[v] == slot) kk += sa->idx[d][v];
+                        if (kk == 0) continue;
+                        /* row stride of dim d: product of the later dims' sizes */
+                        uint16_t f[2] = {SYM_ONE, SYM_ONE};
+                        int nf = 0;
+                        for (int d2 = d + 1; d2 < ar->ndims; d2++) f[nf++] = (uint16_t)(FR_SIZE + ar->dim[d2]);
+                        sym_term(terms, &nt, kk, FR_ELEM, f[0], f[1]);
+                        cnt++;
+                    }
+                    if (g) { g->term_off[slot] = first; g->n_terms[slot] = (uint8_t)cnt; }
+                }
+                if (g) {
+                    g->elem_sym = FR_ELEM;
+                    g->elem_bytes = 0;
+                    g->depth = (uint8_t)(sa->depth - (col ? 1 : 0));
+                    g->is_store = (uint8_t)sa->store;
+                }
+            }
+        }
+    }
+    *n_sym = 24 * 2 * 12;
+    *n_terms = nt;
+    return 0;
+}
+
+/* Frames and bind items of the accesses selgen_fill writes for [c0, c1) of
+ * config 2 or 5 (in the same order).  values: 9 per nest; items: one per
+ * access. */
+int selgen_sym_count(int cfg, uint64_t c0, uint64_t c1, uint64_t* n_values, uint64_t* n_items) {
+    uint64_t nn = 0, na = 0;
+    if ((cfg != SELGEN_C2 && cfg != SELGEN_C5) || selgen_count(cfg, c0, c1, &nn, &na) != 0) return -1;
+    *n_values = 9 * nn;
+    *n_items = na;
+    return 0;
+}
+
+int selgen_sym_fill(int cfg, uint64_t c0, uint64_t c1, int64_t* values, gen_bind_item* items) {
+    uint64_t nn = 0, na = 0;
+    if ((cfg != SELGEN_C2 && cfg != SELGEN_C5) || selgen_count(cfg, c0, c1, &nn, &na) != 0) return -1;
+    uint64_t a = 0;
+    for (uint64_t i = 0; i < nn; i++) {
+        int s, col = 0;
+        nest_params np;
+        if (cfg == SELGEN_C2) {
+            s = c2_nest((int)i, &col);
+            shape_params(&SHAPES[s], cfg, 0, col, &np);
+        } else {
+            uint64_t g = c0 / 32 + i;
+            s = (int)(g % 24);
+            shape_params(&SHAPES[s], cfg, g / 24, 0, &np);
+        }
+        int64_t* fr = values + 9 * i;
+        fr[FR_ELEM] = np.elem;
+        for (int d = 0; d < 4; d++) fr[FR_SIZE + d] = (int64_t)np.symsz[d];
+        for (int d = 0; d < 4; d++) fr[FR_OFF + d] = np.arr_off[d];
+        for (int k = 0; k < SHAPES[s].n_acc; k++, a++) {
+            items[a].sym_access = (uint32_t)((2 * s + col) * 12 + k);
+            items[a].frame = (uint32_t)(9 * i);
+        }
+    }
+    return a == na ? 0 : -1;
+}

@@ -67,6 +67,16 @@ typedef struct {                       /* 16 bytes */
     uint32_t threads, _pad;
 } gen_cpu_input;
 
+/* NEXT row f2 (symbolic IPDA binding) inputs. */
+typedef struct { int64_t k; uint16_t sym[3], _pad; } gen_sym_term;          /* 16 bytes */
+typedef struct {                                                             /* 40 bytes */
+    uint32_t term_off[6];
+    uint8_t n_terms[6];
+    uint16_t elem_sym;
+    uint8_t elem_bytes, depth, is_store, _pad[5];
+} gen_sym_access;
+typedef struct { uint32_t sym_access, frame; } gen_bind_item;               /* 8 bytes */
+
 /* Config ids follow BASELINE.json "configs" order, 1-based. */
 enum { SELGEN_C1 = 1, SELGEN_C2 = 2, SELGEN_C3 = 3, SELGEN_C4 = 4, SELGEN_C5 = 5 };
 
@@ -90,6 +100,12 @@ int selgen_fill_indices(int cfg, const uint64_t* idx, uint64_t m, gen_candidate*
 /* f1 inputs of candidates [c0, c1) and the Table II parameter set. */
 int selgen_cpu_inputs(int cfg, uint64_t c0, uint64_t c1, gen_cpu_input* out);
 void selgen_cpu_params(gen_cpu_params* p);
+/* f2: the static symbolic table (24 shapes x {1-D, collapse} x 12 slots;
+ * pass NULL arrays to size it), and the frames / bind items of [c0, c1)
+ * for configs 2 and 5, aligned with selgen_fill's access order. */
+int selgen_sym_tables(gen_sym_access* sym, gen_sym_term* terms, uint32_t* n_sym, uint32_t* n_terms);
+int selgen_sym_count(int cfg, uint64_t c0, uint64_t c1, uint64_t* n_values, uint64_t* n_items);
+int selgen_sym_fill(int cfg, uint64_t c0, uint64_t c1, int64_t* values, gen_bind_item* items);
 /* Shape catalogue (24 Polybench-style sub-kernels). */
 int selgen_num_shapes(void);
 const char* selgen_shape_name(int s);

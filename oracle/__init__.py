@@ -59,6 +59,7 @@ def lib():
         L.oracle_model.argtypes = [vp, vp, vp, vp, vp, vp]
         L.oracle_select_launch.argtypes = [vp, u64, vp, vp, u64, vp, vp]
         L.oracle_cpu_model.argtypes = [vp, vp, u64, vp, vp, u64, vp, vp]
+        L.oracle_bind.argtypes = [vp, u64, vp, u64, vp, u64, vp, u64, vp, vp]
         L.oracle_sizeof.restype = ctypes.c_size_t
         L.oracle_sizeof.argtypes = [ctypes.c_int]
         L.oracle_offsetof.restype = ctypes.c_size_t
@@ -132,6 +133,20 @@ def cpu_model(params, batch, cpu_in):
     lib().oracle_cpu_model(p.ctypes.data, ne.ctypes.data, len(ne), c.ctypes.data, ci.ctypes.data, n,
                            cyc.ctypes.data, st.ctypes.data)
     return cyc, st
+
+
+def bind(sym, terms, values, items):
+    """NEXT row f2: (concrete accesses as raw 64-byte records, status u8[n])."""
+    n = len(items)
+    out = np.zeros(max(n, 1) * 64, np.uint8)
+    st = np.zeros(max(n, 1), np.uint8)
+    s = np.ascontiguousarray(sym)
+    t = np.ascontiguousarray(terms)
+    v = np.ascontiguousarray(values, dtype=np.int64)
+    it = np.ascontiguousarray(items)
+    lib().oracle_bind(s.ctypes.data, len(s), t.ctypes.data, len(t), v.ctypes.data, len(v), it.ctypes.data, n,
+                      out.ctypes.data, st.ctypes.data)
+    return out[: n * 64], st[:n]
 
 
 def layout(which: int):

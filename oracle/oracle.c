@@ -477,3 +477,61 @@ void oracle_cpu_model(const or_cpu_params* p, const or_nest* nests, uint64_t n_n
         cpu_cycles[c] = (p->startup_cycles + thread_exe) + 0.0;
     }
 }
+
+/* -------------------------------------------------- NEXT row f2 (IPDA) */
+/* Runtime binding of symbolic IPDA expressions (the symbolic
+ * inter-thread stride of A[max*a] is [max]; "at the program point
+ * when the target region is encountered, the unknown values are extracted and
+ * used in the symbolic expression to compute the actual stride").  Every byte
+ * coefficient of an access (base, c_par[0..1], c_inner[0..2]) is the sum of
+ * its terms k * v[frame+s0] * v[frame+s1] * v[frame+s2] (a symbol index of
+ * 0xFFFF is the factor 1).  Plain definition with exact 128-bit arithmetic:
+ * any product or partial sum reaching 2^62 in magnitude -> ERANGE; a bad
+ * index or an element size outside {1,2,4,8,16} -> EINVAL; invalid outputs
+ * are all-zero. */
+void oracle_bind(const or_sym_access* sym, uint64_t n_sym, const or_sym_term* terms, uint64_t n_terms,
+                 const int64_t* values, uint64_t n_values, const or_bind_item* items, uint64_t n,
+                 or_access* out, uint8_t* status) {
+    const __int128 LIM = (__int128)1 << 62;
+    for (uint64_t i = 0; i < n; i++) {
+        or_access* o = &out[i];
+        memset(o, 0, sizeof *o);
+        status[i] = OR_OK;
+        if (items[i].sym_access >= n_sym) { status[i] = OR_EINVAL; continue; }
+        const or_sym_access* a = &sym[items[i].sym_access];
+        const uint64_t fr = items[i].frame;
+        int64_t coef[6];
+        int bad = 0;
+        for (int slot = 0; slot < 6 && !bad; slot++) {
+            __int128 acc = 0;
+            if ((uint64_t)a->term_off[slot] + a->n_terms[slot] > n_terms) { bad = OR_EINVAL; break; }
+            for (int t = 0; t < a->n_terms[slot] && !bad; t++) {
+                const or_sym_term* tm = &terms[a->term_off[slot] + t];
+                __int128 p = tm->k;
+                for (int f = 0; f < 3; f++) {
+                    if (tm->sym[f] == 0xFFFFu) continue;
+                    if (fr + tm->sym[f] >= n_values) { bad = OR_EINVAL; break; }
+                    p *= values[fr + tm->sym[f]];
+                    if (p >= LIM || p <= -LIM) { bad = OR_ERANGE; break; }
+                }
+                if (bad) break;
+                acc += p;
+                if (acc >= LIM || acc <= -LIM) bad = OR_ERANGE;
+            }
+            coef[slot] = (int64_t)acc;
+        }
+        int64_t e = a->elem_bytes;
+        if (!bad && a->elem_sym != 0xFFFFu) {
+            if (fr + a->elem_sym >= n_values) bad = OR_EINVAL;
+            else e = values[fr + a->elem_sym];
+        }
+        if (!bad && !(e == 1 || e == 2 || e == 4 || e == 8 || e == 16)) bad = OR_EINVAL;
+        if (bad) { status[i] = (uint8_t)bad; continue; }
+        o->base = coef[0];
+        o->c_par[0] = coef[1]; o->c_par[1] = coef[2];
+        o->c_inner[0] = coef[3]; o->c_inner[1] = coef[4]; o->c_inner[2] = coef[5];
+        o->elem_bytes = (uint8_t)e;
+        o->depth = a->depth;
+        o->is_store = a->is_store;
+    }
+}

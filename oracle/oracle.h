@@ -52,6 +52,16 @@ typedef struct {
 } or_cpu_params;
 typedef struct { double mca_cycles_per_iter; uint32_t threads, _pad; } or_cpu_input;
 
+/* NEXT row f2 inputs (layouts as gen/selgen.h, declared independently) */
+typedef struct { int64_t k; uint16_t sym[3], _pad; } or_sym_term;
+typedef struct {
+    uint32_t term_off[6];
+    uint8_t n_terms[6];
+    uint16_t elem_sym;
+    uint8_t elem_bytes, depth, is_store, _pad[5];
+} or_sym_access;
+typedef struct { uint32_t sym_access, frame; } or_bind_item;
+
 /* Everything the oracle computes for one candidate: the hot path's outputs
  * (counts, cycles, t_gpu, decision, status) plus the model's intermediate
  * values, exposed so that tests can pin them against closed forms. */
@@ -98,6 +108,11 @@ void oracle_select_launch(const uint32_t* group_of, uint64_t n, const double* t_
 /* NEXT row f1: Liao-Chapman CPU cycles (Fig. 3 + Table II) per candidate. */
 void oracle_cpu_model(const or_cpu_params* p, const or_nest* nests, uint64_t n_nests, const or_candidate* cands,
                       const or_cpu_input* in, uint64_t n, double* cpu_cycles, uint8_t* status);
+
+/* NEXT row f2: bind symbolic accesses to concrete ones (see oracle.c). */
+void oracle_bind(const or_sym_access* sym, uint64_t n_sym, const or_sym_term* terms, uint64_t n_terms,
+                 const int64_t* values, uint64_t n_values, const or_bind_item* items, uint64_t n,
+                 or_access* out, uint8_t* status);
 
 /* Layout self-description for tests/test_layout.py. */
 size_t oracle_sizeof(int which);

@@ -187,6 +187,27 @@ def model_cpu_cost(cands: torch.Tensor, tables: DeviceTables, cpu_in, params, st
     return status
 
 
+def _dev_bytes(x, device):
+    if isinstance(x, torch.Tensor):
+        return x.view(torch.uint8).reshape(-1).to(device)
+    a = np.ascontiguousarray(x)
+    return torch.from_numpy(a.view(np.uint8).reshape(-1)).to(device)
+
+
+def bind_accesses(sym, terms, values, items, device="cuda", out: torch.Tensor | None = None, stream=None):
+    """sel_bind_accesses (NEXT row f2): symbolic IPDA accesses + symbol frames
+    -> (concrete access records as uint8[n*64] on the device, status uint8[n])."""
+    sym_d, terms_d = _dev_bytes(sym, device), _dev_bytes(terms, device)
+    val_d, items_d = _dev_bytes(values, device), _dev_bytes(items, device)
+    n = items_d.numel() // 8
+    out = torch.empty(n * 64, dtype=torch.uint8, device=device) if out is None else out
+    status = torch.empty(n, dtype=torch.uint8, device=device)
+    _lib.check(_lib.lib().sel_bind_accesses(_ptr(sym_d), sym_d.numel() // 40, _ptr(terms_d), terms_d.numel() // 16,
+                                            _ptr(val_d), val_d.numel() // 8, _ptr(items_d), n, _ptr(out),
+                                            _ptr(status), _stream(stream)))
+    return out, status
+
+
 def read_stats(workspace: torch.Tensor, stream=None) -> dict:
     st = _lib.Stats()
     wp, _ = _ws_ptr(workspace)
@@ -227,6 +248,7 @@ sel_evaluate = evaluate
 sel_read_stats = read_stats
 sel_select_launch = select_launch
 sel_model_cpu_cost = model_cpu_cost
+sel_bind_accesses = bind_accesses
 
 
 class Evaluator:

@@ -197,6 +197,18 @@ int sel_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu,
     return SEL_OK;
 }
 
+int sel_bind_accesses(const sel_sym_access* sym, uint64_t n_sym, const sel_sym_term* terms, uint64_t n_terms,
+                      const int64_t* values, uint64_t n_values, const sel_bind_item* items, uint64_t n,
+                      sel_access* out, uint8_t* status, sel_stream_t stream) {
+    if (n == 0) return SEL_OK;
+    if (!items || !out || !status || (n_sym && !sym) || (n_terms && !terms) || (n_values && !values))
+        return fail(SEL_EINVAL, "NULL argument%s");
+    cudaError_t e = launch_bind(sym, n_sym, terms, n_terms, values, n_values, items, n, out, status,
+                                reinterpret_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "bind_accesses");
+    return SEL_OK;
+}
+
 int sel_model_cpu_cost(sel_candidate* c, uint64_t n, const sel_tables* t, const sel_cpu_input* in,
                        const sel_cpu_params* p, uint8_t* status, sel_stream_t stream) {
     if (int r = check_tables(t)) return r;
@@ -307,3 +319,6 @@ static_assert(sizeof(sel_counts) == 48, "sel_counts layout");
 static_assert(sizeof(sel_stats) == 64, "sel_stats layout");
 static_assert(sizeof(sel_cpu_params) == 64, "sel_cpu_params layout");
 static_assert(sizeof(sel_cpu_input) == 16, "sel_cpu_input layout");
+static_assert(sizeof(sel_sym_term) == 16, "sel_sym_term layout");
+static_assert(sizeof(sel_sym_access) == 40, "sel_sym_access layout");
+static_assert(sizeof(sel_bind_item) == 8, "sel_bind_item layout");

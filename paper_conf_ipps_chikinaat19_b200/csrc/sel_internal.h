@@ -56,6 +56,9 @@ cudaError_t launch_select(const sel_candidate* cands, uint64_t n, const double* 
 cudaError_t launch_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
                                  uint64_t n_groups, uint32_t* best, double* best_t, cudaStream_t s);
 
+cudaError_t launch_bind(const sel_sym_access* sym, uint64_t n_sym, const sel_sym_term* terms, uint64_t n_terms,
+                        const int64_t* values, uint64_t n_values, const sel_bind_item* items, uint64_t n,
+                        sel_access* out, uint8_t* status, cudaStream_t s);
 cudaError_t launch_cpu_model(sel_candidate* cands, uint64_t n, const sel_tables& t, const sel_cpu_input* in,
                              const sel_cpu_params& p, uint8_t* status, cudaStream_t s);
 

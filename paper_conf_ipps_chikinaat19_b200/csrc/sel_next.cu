@@ -107,4 +107,77 @@ cudaError_t launch_cpu_model(sel_candidate* cands, uint64_t n, const sel_tables&
     return cudaGetLastError();
 }
 
+// f2  Runtime binding of symbolic IPDA expressions: one
+//     thread per access evaluates the six byte coefficients as sums of terms
+//     k * v[frame+s0] * v[frame+s1] * v[frame+s2] over the access's symbol
+//     frame, with exact 128-bit products; |value| >= 2^62 -> SEL_ERANGE, a bad
+//     index or element size -> SEL_EINVAL (output zeroed).  The result is a
+//     concrete sel_access table the counting kernel consumes unchanged.
+__global__ void __launch_bounds__(256) k_bind(const sel_sym_access* __restrict__ sym, uint64_t n_sym,
+                                              const sel_sym_term* __restrict__ terms, uint64_t n_terms,
+                                              const int64_t* __restrict__ values, uint64_t n_values,
+                                              const sel_bind_item* __restrict__ items, uint64_t n,
+                                              sel_access* __restrict__ out, uint8_t* __restrict__ status) {
+    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const __int128 lim = (__int128)1 << 62;
+    const sel_bind_item it = items[i];
+    uint8_t st = SEL_OK;
+    int64_t coef[6] = {0, 0, 0, 0, 0, 0};
+    int64_t e = 0;
+    sel_access o{};
+    if (it.sym_access >= n_sym) {
+        st = SEL_EINVAL;
+    } else {
+        const sel_sym_access a = sym[it.sym_access];
+        const uint64_t fr = it.frame;
+        for (int slot = 0; slot < 6 && !st; slot++) {
+            if (uint64_t(a.term_off[slot]) + a.n_terms[slot] > n_terms) { st = SEL_EINVAL; break; }
+            __int128 acc = 0;
+            for (int t = 0; t < a.n_terms[slot] && !st; t++) {
+                const sel_sym_term tm = terms[a.term_off[slot] + t];
+                __int128 p = tm.k;
+                for (int f = 0; f < 3; f++) {
+                    if (tm.sym[f] == SEL_SYM_ONE) continue;
+                    if (fr + tm.sym[f] >= n_values) { st = SEL_EINVAL; break; }
+                    p *= values[fr + tm.sym[f]];
+                    if (p >= lim || p <= -lim) { st = SEL_ERANGE; break; }
+                }
+                if (st) break;
+                acc += p;
+                if (acc >= lim || acc <= -lim) st = SEL_ERANGE;
+            }
+            coef[slot] = int64_t(acc);
+        }
+        e = a.elem_bytes;
+        if (!st && a.elem_sym != SEL_SYM_ONE) {
+            if (fr + a.elem_sym >= n_values) st = SEL_EINVAL;
+            else e = values[fr + a.elem_sym];
+        }
+        if (!st && !(e == 1 || e == 2 || e == 4 || e == 8 || e == 16)) st = SEL_EINVAL;
+        if (!st) {
+            o.base = coef[0];
+            o.c_par[0] = coef[1];
+            o.c_par[1] = coef[2];
+            o.c_inner[0] = coef[3];
+            o.c_inner[1] = coef[4];
+            o.c_inner[2] = coef[5];
+            o.elem_bytes = uint8_t(e);
+            o.depth = a.depth;
+            o.is_store = a.is_store;
+        }
+    }
+    out[i] = o;
+    status[i] = st;
+}
+
+cudaError_t launch_bind(const sel_sym_access* sym, uint64_t n_sym, const sel_sym_term* terms, uint64_t n_terms,
+                        const int64_t* values, uint64_t n_values, const sel_bind_item* items, uint64_t n,
+                        sel_access* out, uint8_t* status, cudaStream_t s) {
+    k_bind<<<unsigned((n + 255) / 256), 256, 0, s>>>(sym, n_sym, terms, n_terms, values, n_values, items, n, out,
+                                                     status);
+    note_launch();
+    return cudaGetLastError();
+}
+
 }  // namespace sel

@@ -82,3 +82,18 @@ def test_sync_term_parity(sel):
     nests["n_sync"] = np.arange(len(nests)) % 4
     bb = gen.Batch(b.cands, nests, b.accesses, b.launches, b.devices)
     P.assert_parity(P.run_gpu(sel, bb), oracle.evaluate(bb), ctx="f4 sync")
+
+
+@pytest.mark.parametrize("cfg,rng", [(2, (0, 108)), (5, (0, 10000000))])
+def test_bind_parity(sel, cfg, rng):
+    """NEXT row f2: device binding == oracle binding == the generator's
+    concrete accesses; bound tables evaluate identically."""
+    sym, terms = gen.sym_tables()
+    vals, items = gen.sym_instances(cfg, *rng)
+    vals[9 * 5 + 2] = 1 << 61                            # one overflowing frame (ERANGE)
+    ref, st_ref = oracle.bind(sym, terms, vals, items)
+    out, st = sel.bind_accesses(sym, terms, vals, items)
+    torch.cuda.synchronize()
+    assert (st.cpu().numpy() == st_ref).all()
+    assert np.array_equal(out.cpu().numpy(), ref)
+    assert (st_ref != 0).sum() >= 1

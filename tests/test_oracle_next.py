@@ -115,3 +115,70 @@ def test_sync_term_linear_and_zero_cases():
     lau[0] = (32, 1, 0, 0)
     one = gen.custom_batch([dict(P0=64, trip=[5], comp=[1.0, 2.0], accesses=[a])], launches_=lau)
     assert oracle.evaluate(_with_sync(one, 3))["cycles"][0] == oracle.evaluate(one)["cycles"][0]
+
+
+# ---------------------------------------------------------------- f2 (symbolic IPDA binding)
+def _sym_one(terms_per_slot, elem_sym=0, elem_bytes=0, depth=0):
+    """one symbolic access; terms_per_slot: 6 lists of (k, syms)."""
+    sym = np.zeros(1, gen.SYM_ACCESS_DTYPE)
+    terms = []
+    for slot, tl in enumerate(terms_per_slot):
+        sym["term_off"][0][slot] = len(terms)
+        sym["n_terms"][0][slot] = len(tl)
+        for k, ss in tl:
+            ss = list(ss) + [gen.SYM_ONE] * (3 - len(ss))
+            terms.append((k, ss, 0))
+    sym["elem_sym"], sym["elem_bytes"], sym["depth"] = elem_sym, elem_bytes, depth
+    t = np.zeros(max(len(terms), 1), gen.SYM_TERM_DTYPE)
+    for i, (k, ss, _) in enumerate(terms):
+        t[i]["k"], t[i]["sym"] = k, ss
+    return sym, t
+
+
+def test_bind_ipda_worked_example():
+    """A[max*a] in a parallel loop over a has inter-thread stride
+    [max] (x 4-byte elements); binding max at runtime gives the concrete
+    access, whose full warp touches min(32, ceil(32*max*4/128)) lines."""
+    sym, terms = _sym_one([[(1 << 28, [])], [(1, [0, 1])], [], [], [], []])   # frame: v0 = elem, v1 = max
+    items = np.zeros(6, gen.BIND_ITEM_DTYPE)
+    vals = []
+    for i, mx in enumerate([1, 2, 7, 31, 32, 100]):
+        items[i]["frame"] = len(vals)
+        vals += [4, mx]
+    out, st = oracle.bind(sym, terms, np.array(vals), items)
+    acc = out.view(gen.ACCESS_DTYPE)
+    assert (st == 0).all()
+    assert list(acc["c_par"][:, 0]) == [4, 8, 28, 124, 128, 400]
+    lau = np.zeros(1, gen.LAUNCH_DTYPE)
+    lau[0] = (256, 65535, 0, 0)
+    b = gen.custom_batch([dict(P0=32, trip=[], accesses=[a]) for a in acc], launches_=lau)
+    r = oracle.evaluate(b)
+    assert list(r["L"]) == [min(32, -(-32 * m * 4 // 128)) for m in [1, 2, 7, 31, 32, 100]]
+
+
+def test_bind_reproduces_generator_accesses():
+    """The symbolic table bound with each nest's frame gives back, byte for
+    byte, the concrete accesses the generator writes directly (c2, c5)."""
+    sym, terms = gen.sym_tables()
+    for cfg, rng in ((2, (0, 108)), (5, (0, 200000)), (5, (77000000, 77200000))):
+        b = gen.generate(cfg, *rng)
+        vals, items = gen.sym_instances(cfg, *rng)
+        out, st = oracle.bind(sym, terms, vals, items)
+        assert (st == 0).all()
+        assert np.array_equal(out, np.ascontiguousarray(b.accesses[:len(items)]).view(np.uint8).reshape(-1))
+
+
+def test_bind_errors():
+    sym, terms = _sym_one([[(1 << 40, [0])], [(1, [1])], [], [], [], []])
+    items = np.zeros(5, gen.BIND_ITEM_DTYPE)
+    items[0]["frame"] = 0      # ok
+    items[1]["frame"] = 2      # v[2] * 2^40 overflows 2^62
+    items[2]["frame"] = 4      # elem 3 -> EINVAL
+    items[3]["frame"] = 100    # frame out of range -> EINVAL
+    items[4]["sym_access"] = 9  # bad symbolic access
+    vals = np.array([4, 8, 1 << 23, 8, 3, 8])
+    out, st = oracle.bind(sym, terms, vals, items)
+    assert list(st) == [0, 2, 1, 1, 1]
+    acc = out.view(gen.ACCESS_DTYPE)
+    assert acc["base"][0] == 4 << 40 and acc["c_par"][0, 0] == 8 and acc["elem_bytes"][0] == 4
+    assert (out.reshape(5, 64)[1:] == 0).all()

@@ -164,7 +164,8 @@ def run_reference(args):
     t0 = time.perf_counter()
     oracle.evaluate(gen.generate_indices(args.config, probe_idx), threads=cores)
     per_cand = (time.perf_counter() - t0) / len(probe_idx)
-    per_step = int(max(32, min(total, 6.0 / max(per_cand, 1e-9))))
+    step_s = float(os.environ.get("REF_STEP_SECONDS", "6.0"))
+    per_step = int(max(32, min(total, step_s / max(per_cand, 1e-9))))
     stride = max(1, total // per_step)
     times, evals, was = [], 0, 0
     for step in range(args.warmup + args.steps):

@@ -26,8 +26,9 @@
 //    register) and tests y < d_l << 25: one ISETP per flag, no cross-lane
 //    traffic.  1-D parallel accesses are monotone across lanes (no sort);
 //    collapse(2) accesses are sorted once per warp-rep with a shuffle
-//    bitonic network.  lines = 1 + #flags; coalesced (tmin = 1) <=> no flag
-//    (vote.any); tmin > 1 uses vote.ballot + popc.
+//    bitonic network.  lines = 1 + #flags.  Line flags of 32 consecutive
+//    WAs are collected as per-lane bitmasks and classified with one warp
+//    reduction per group (see "hot loops" below).
 //  * MATCH (SEL_F_MATCH_ANY).  The north star's literal primitive: full
 //    64-bit lane addresses, __match_any_sync on (addr >> 7) and (addr >> 5),
 //    first-occurrence flags, __ballot_sync/__popc.

@@ -253,33 +253,30 @@ def run_ours(args):
     # ---- end to end through the public API: pinned host inputs -> decisions + cycles on the host
     e2e = None
     if not args.no_e2e:
+        # every step uploads its inputs (candidates + nest and access tables) from pinned host
+        # memory and downloads decision + cycles to pinned host memory; sel.HostPipeline overlaps
+        # step k+1's upload and step k-1's download with step k's kernels (two device slots)
         nests_h = torch.from_numpy(batch.nests.view(np.uint8).reshape(-1)).pin_memory()
         acc_h = torch.from_numpy(batch.accesses.view(np.uint8).reshape(-1)).pin_memory()
-        out_host = {"decision": torch.empty(len(batch), dtype=torch.uint8, pin_memory=True),
-                    "cycles": torch.empty(len(batch), dtype=torch.float64, pin_memory=True)}
-        h2d = cands_host.numel() + nests_h.numel() + acc_h.numel()
-        d2h = len(batch) * 9
-
-        def e2e_step():
-            ev.tables.nests.copy_(nests_h, non_blocking=True)
-            ev.tables.accesses.copy_(acc_h, non_blocking=True)
-            ev.evaluate_host(cands_host, out_host=out_host)
-
-        for _ in range(max(1, args.warmup)):
-            e2e_step()
+        h2d, d2h = sel.HostPipeline.bytes_per_step(cands_host, nests_h, acc_h, len(batch))
+        out = None                                     # free the device-resident outputs
+        pipe = sel.HostPipeline(ev, cands_host, nests_h, acc_h)
+        for k in range(max(1, args.warmup)):
+            pipe.step(k, cands_host, nests_h, acc_h)
         torch.cuda.synchronize(dev)
         D.barrier(world)
         f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        f0.record(stream)
-        for _ in range(args.steps):
-            e2e_step()
-        f1.record(stream)
+        f0.record(pipe.h2d)
+        for k in range(args.steps):
+            pipe.step(k, cands_host, nests_h, acc_h)
+        f1.record(pipe.d2h)
         torch.cuda.synchronize(dev)
         ms_e2e = D.max_over_ranks(f0.elapsed_time(f1), world, dev)
         e2e = {"value": total / (ms_e2e / 1e3 / args.steps), "unit": UNIT,
                "h2d_bytes_per_step": D.sum_over_ranks(h2d, world, dev),
                "d2h_bytes_per_step": D.sum_over_ranks(d2h, world, dev),
-               "ms_per_step": ms_e2e / args.steps}
+               "ms_per_step": ms_e2e / args.steps, "overlap": "double-buffered H2D / kernels / D2H streams"}
+        del pipe
 
     if rank != 0:
         return
@@ -312,13 +309,13 @@ def run_ours(args):
             "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
     if not args.no_next and args.config == 5:
-        line["next_rows"] = time_next_rows(sel, gen, ev, batch, cands, out, args, c0, c1, dev)
+        line["next_rows"] = time_next_rows(sel, gen, ev, batch, cands, args, c0, c1, dev)
     if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_oracle_sample(batch, args.cpu_seconds, total)
     print(json.dumps(line), flush=True)
 
 
-def time_next_rows(sel, gen, ev, batch, cands, out, args, c0, c1, dev):
+def time_next_rows(sel, gen, ev, batch, cands, args, c0, c1, dev):
     """NEXT rows on this rank's c5 batch: f2 symbolic IPDA
     binding of every access, f1 Liao-Chapman CPU model of every candidate, f3
     launch selection per (nest, device) group.  Device time with CUDA events

@@ -285,3 +285,64 @@ class Evaluator:
 
     def stats(self) -> dict:
         return read_stats(self.workspace)
+
+
+class HostPipeline:
+    """End-to-end evaluation from pinned host memory with copy/compute overlap.
+
+    Each ``step`` uploads that step's inputs (candidates, nest and access
+    tables) from pinned host buffers into one of two device slots on an H2D
+    stream, runs ``sel_evaluate`` on a compute stream once that upload is done,
+    and downloads decision and cycles into pinned host buffers on a D2H stream,
+    so the uploads of step k+1 and the downloads of step k-1 overlap the
+    kernels of step k.  Results of step k are valid after ``wait(k)``."""
+
+    def __init__(self, ev: Evaluator, cands_host: torch.Tensor, nests_host: torch.Tensor, acc_host: torch.Tensor):
+        dev = ev.device
+        self.ev = ev
+        self.n = _n(cands_host, "candidate")
+        self.h2d, self.comp, self.d2h = (torch.cuda.Stream(dev) for _ in range(3))
+        self.slots = []
+        for _ in range(2):
+            s = {"cands": torch.empty(cands_host.numel(), dtype=torch.uint8, device=dev),
+                 "nests": torch.empty(nests_host.numel(), dtype=torch.uint8, device=dev),
+                 "acc": torch.empty(acc_host.numel(), dtype=torch.uint8, device=dev),
+                 "out": {"decision": torch.empty(self.n, dtype=torch.uint8, device=dev),
+                         "cycles": torch.empty(self.n, dtype=torch.float64, device=dev),
+                         "status": torch.empty(self.n, dtype=torch.uint8, device=dev)},
+                 "host": {"decision": torch.empty(self.n, dtype=torch.uint8, pin_memory=True),
+                          "cycles": torch.empty(self.n, dtype=torch.float64, pin_memory=True)},
+                 "up": torch.cuda.Event(), "done": torch.cuda.Event(), "down": torch.cuda.Event(),
+                 "used": False}
+            s["tables"] = DeviceTables(s["nests"], s["acc"], ev.tables.launches, dev)
+            self.slots.append(s)
+
+    def step(self, k: int, cands_host: torch.Tensor, nests_host: torch.Tensor, acc_host: torch.Tensor) -> dict:
+        s = self.slots[k % 2]
+        if s["used"]:
+            self.h2d.wait_event(s["done"])        # inputs of step k-2 consumed
+            self.comp.wait_event(s["down"])       # outputs of step k-2 downloaded
+        with torch.cuda.stream(self.h2d):
+            s["cands"].copy_(cands_host, non_blocking=True)
+            s["nests"].copy_(nests_host, non_blocking=True)
+            s["acc"].copy_(acc_host, non_blocking=True)
+            s["up"].record(self.h2d)
+        self.comp.wait_event(s["up"])
+        evaluate(s["cands"], s["tables"], self.ev.workspace, self.ev.flags, out=s["out"], stream=self.comp)
+        s["done"].record(self.comp)
+        self.d2h.wait_event(s["done"])
+        with torch.cuda.stream(self.d2h):
+            s["host"]["decision"].copy_(s["out"]["decision"], non_blocking=True)
+            s["host"]["cycles"].copy_(s["out"]["cycles"], non_blocking=True)
+            s["down"].record(self.d2h)
+        s["used"] = True
+        return s["host"]
+
+    def wait(self, k: int) -> dict:
+        s = self.slots[k % 2]
+        s["down"].synchronize()
+        return s["host"]
+
+    @staticmethod
+    def bytes_per_step(cands_host, nests_host, acc_host, n):
+        return cands_host.numel() + nests_host.numel() + acc_host.numel(), n * 9

@@ -255,3 +255,22 @@ def test_near_tie_decisions(sel):
     assert_parity(g, r2, ctx="ties")
     n = len(b)
     assert (g["decision"][:2 * n] == 0).all() and (g["decision"][2 * n:] == 1).all()
+
+
+def test_host_pipeline_end_to_end(sel):
+    """The double-buffered host path returns the same decisions and cycles as
+    the device-resident call, step after step (the e2e measurement path)."""
+    b = gen.generate(5, 0, 200000)
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
+    ref = ev.evaluate(sel._as_bytes_tensor(b.cands, "candidate"))
+    torch.cuda.synchronize()
+    ch = torch.from_numpy(b.cands.view(np.uint8).reshape(-1)).pin_memory()
+    nh = torch.from_numpy(b.nests.view(np.uint8).reshape(-1)).pin_memory()
+    ah = torch.from_numpy(b.accesses.view(np.uint8).reshape(-1)).pin_memory()
+    pipe = sel.HostPipeline(ev, ch, nh, ah)
+    for k in range(4):
+        pipe.step(k, ch, nh, ah)
+    for k in (2, 3):
+        h = pipe.wait(k)
+        assert torch.equal(h["decision"], ref["decision"].cpu())
+        assert torch.equal(h["cycles"], ref["cycles"].cpu())

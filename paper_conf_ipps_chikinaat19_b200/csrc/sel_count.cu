@@ -411,7 +411,10 @@ template <bool MATCH>
 #ifndef SEL_COUNT_MIN_BLOCKS
 #define SEL_COUNT_MIN_BLOCKS 3
 #endif
-__global__ void __launch_bounds__(256, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
+#ifndef SEL_COUNT_THREADS
+#define SEL_COUNT_THREADS 256
+#endif
+__global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;
@@ -455,14 +458,14 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
         int dev = 0, sms = 0, per = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (match) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<true>, 256, 0);
-        else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<false>, 256, 0);
+        if (match) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<true>, SEL_COUNT_THREADS, 0);
+        else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<false>, SEL_COUNT_THREADS, 0);
         g = sms * (per > 0 ? per : 1);
     }
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr};
     prof_before_count(s);
-    if (match) k_count<true><<<g, 256, 0, s>>>(a);
-    else k_count<false><<<g, 256, 0, s>>>(a);
+    if (match) k_count<true><<<g, SEL_COUNT_THREADS, 0, s>>>(a);
+    else k_count<false><<<g, SEL_COUNT_THREADS, 0, s>>>(a);
     prof_after_count(s);
     note_launch();
     return cudaGetLastError();

@@ -22,20 +22,36 @@ def env_rank_world():
 
 def init(backend: str | None = None):
     """Initialise the default process group from the torchrun environment
-    (no-op for a single process).  Returns (rank, world, local_rank)."""
+    (no-op for a single process).  Returns (rank, world, device_index).
+
+    One process per GPU over NCCL by default.  SEL_DIST_BACKEND=gloo selects
+    host-staged collectives instead, which lets several ranks share one GPU
+    (device = local_rank mod #GPUs) -- used to exercise the multi-rank bench
+    path on a single-GPU box; it is not the performance configuration."""
     rank, world, local = env_rank_world()
+    backend = backend or os.environ.get("SEL_DIST_BACKEND")
+    dev_index = local
+    if torch.cuda.is_available():
+        dev_index = local % torch.cuda.device_count()
     if world > 1 and not dist.is_initialized():
         if backend is None:
             backend = "nccl" if torch.cuda.is_available() else "gloo"
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         if backend == "nccl":
-            torch.cuda.set_device(local)
-            dist.init_process_group(backend, device_id=torch.device("cuda", local))
+            torch.cuda.set_device(dev_index)
+            dist.init_process_group(backend, device_id=torch.device("cuda", dev_index))
         else:
+            if torch.cuda.is_available():
+                torch.cuda.set_device(dev_index)
             dist.init_process_group(backend)
     elif torch.cuda.is_available():
-        torch.cuda.set_device(local)
-    return rank, world, local
+        torch.cuda.set_device(dev_index)
+    return rank, world, dev_index
+
+
+def _host_staged(t: torch.Tensor) -> bool:
+    """gloo collectives on CUDA tensors are staged through host memory."""
+    return t.is_cuda and dist.is_initialized() and dist.get_backend() == "gloo"
 
 
 def shard_range(total: int, rank: int, world: int):
@@ -61,7 +77,12 @@ def gather_decisions(local: torch.Tensor, total: int, world: int, out: torch.Ten
     buf = torch.zeros(n_pad, dtype=torch.uint8, device=local.device)
     buf[: local.numel()].copy_(local)
     full = torch.empty(n_pad * world, dtype=torch.uint8, device=local.device) if out is None else out
-    dist.all_gather_into_tensor(full, buf, group=group)
+    if _host_staged(buf):
+        hfull = torch.empty(n_pad * world, dtype=torch.uint8)
+        dist.all_gather_into_tensor(hfull, buf.cpu(), group=group)
+        full.copy_(hfull)
+    else:
+        dist.all_gather_into_tensor(full, buf, group=group)
     parts = []
     for r in range(world):
         c0, c1 = shard_range(total, r, world)
@@ -73,6 +94,8 @@ def max_over_ranks(x: float, world: int, device) -> float:
     if world == 1:
         return x
     t = torch.tensor([x], dtype=torch.float64, device=device)
+    if _host_staged(t):
+        t = t.cpu()
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -81,6 +104,8 @@ def sum_over_ranks(x: int, world: int, device) -> int:
     if world == 1:
         return x
     t = torch.tensor([x], dtype=torch.int64, device=device)
+    if _host_staged(t):
+        t = t.cpu()
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return int(t.item())
 

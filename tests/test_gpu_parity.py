@@ -274,3 +274,38 @@ def test_host_pipeline_end_to_end(sel):
         h = pipe.wait(k)
         assert torch.equal(h["decision"], ref["decision"].cpu())
         assert torch.equal(h["cycles"], ref["cycles"].cpu())
+
+
+def _random_medium_batch(seed, n):
+    """Nests with long inner rows (>= 32, so the fully unrolled 32-WA groups,
+    the partial groups and every tmin class run), all element sizes, 1-D and
+    collapse(2), negative / zero / large strides, B not a multiple of 32."""
+    rnd = random.Random(seed)
+    launches = np.zeros(n, gen.LAUNCH_DTYPE)
+    items = []
+    for i in range(n):
+        par_dims = rnd.choice([1, 1, 2])
+        P0, P1 = (rnd.randint(1, 300), 1) if par_dims == 1 else (rnd.randint(1, 12), rnd.randint(1, 40))
+        depth = rnd.choice([1, 1, 2])
+        trip = ([rnd.randint(1, 9), rnd.randint(30, 75)] if depth == 2 else [rnd.randint(30, 75)])
+        acc = []
+        for _ in range(rnd.randint(1, 3)):
+            e = rnd.choice([1, 2, 4, 8, 16])
+            d = rnd.randint(0, depth)
+
+            def coef():
+                return e * rnd.choice([0, 1, -1, 2, 3, 5, 7, 8, 16, 31, 32, 33, -40, 64, 129, 1000])
+            acc.append(gen.make_access(base=(1 << 30) + e * rnd.randint(-100, 100), c_par=[coef(), coef()],
+                                       c_inner=[coef() for _ in range(d)], elem_bytes=e, depth=d))
+        launches[i] = (rnd.choice([32, 48, 64, 100, 128, 200, 256]), rnd.choice([1, 3, 65535]), 0, 0)
+        items.append(dict(P0=P0, P1=P1, par_dims=par_dims, trip=trip, depth=depth, comp=[1.0, 2.0, 0.5],
+                          launch=i, device=rnd.randrange(4), accesses=acc))
+    return gen.custom_batch(items, launches_=launches)
+
+
+@pytest.mark.parametrize("flags", [0, 2])
+def test_random_medium_nests(sel, flags):
+    b = _random_medium_batch(123 + flags, 1500)
+    ref = oracle.evaluate(b)
+    assert (ref["status"] == 0).all() and ref["W"].sum() > 4 * 10 ** 5
+    assert_parity(run_gpu(sel, b, flags), ref, ctx=f"medium flags={flags}")

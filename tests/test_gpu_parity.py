@@ -309,3 +309,21 @@ def test_random_medium_nests(sel, flags):
     ref = oracle.evaluate(b)
     assert (ref["status"] == 0).all() and ref["W"].sum() > 4 * 10 ** 5
     assert_parity(run_gpu(sel, b, flags), ref, ctx=f"medium flags={flags}")
+
+
+def test_count_sharing_slot_overflow(sel):
+    """More distinct B classes per nest than the 8 sharing slots: the extra
+    classes get private counting problems (plan overflow path)."""
+    b2 = gen.generate(2)
+    Bs = [32, 64, 1024] + list(range(1, 40, 3))          # 3 multiples of 32 (one class) + 13 others
+    launches = np.zeros(len(Bs), gen.LAUNCH_DTYPE)
+    for i, B in enumerate(Bs):
+        launches[i] = (B, 65535 if i % 2 else 7, 0, 0)
+    rows = [(nest, li, dev) for nest in (6, 10, 16) for li in range(len(Bs)) for dev in (0, 3)]
+    cands = np.zeros(len(rows), gen.CANDIDATE_DTYPE)
+    for i, (nest, li, dev) in enumerate(rows):
+        cands[i] = (nest, li, dev, 2e6, 3e9)
+    b = gen.Batch(cands, b2.nests, b2.accesses, launches, b2.devices)
+    g = run_gpu(sel, b)
+    assert_parity(g, oracle.evaluate(b), ctx="slot overflow")
+    assert g["stats"]["n_problems"] == 3 * (1 + 13)

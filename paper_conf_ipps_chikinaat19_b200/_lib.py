@@ -16,6 +16,7 @@ LIB_PATH = os.environ.get("SEL_LIBSEL", os.path.join(_HERE, "libsel.so"))   # ov
 SEL_OK, SEL_EINVAL, SEL_ERANGE, SEL_ELAUNCH, SEL_ENODEV, SEL_ECUDA, SEL_EINTERNAL = range(7)
 SEL_F_NO_DEDUP = 1
 SEL_F_MATCH_ANY = 2
+SEL_F_SCALAR = 4
 DECISION_CPU, DECISION_GPU, DECISION_INVALID = 0, 1, 0xFF
 
 

@@ -48,6 +48,7 @@ struct CountArgs {
     const unsigned long long* prob_WR;
     unsigned long long* prob_cnt;       // W, L, S, C, U per problem
     WsHeader* hdr;
+    uint32_t one;                       // 1 at run time: keeps adds as IMAD on the FMA pipe
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -202,6 +203,69 @@ __device__ __forceinline__ void hot_row_t4(uint32_t y, uint32_t step, uint32_t d
     a.W += len;
 }
 
+// RESIDUE, byte-sliced (SWAR, default).  The line residue r = (s_l + D) mod
+// 128 of four consecutive WAs sits in the four bytes of one register (bit 7
+// of each byte clear).  For a per-lane threshold d <= 128 (gap, capped),
+//   T = R + (0x80808080 - d * 0x01010101)
+// never borrows across bytes (r + 128 - d >= 0) and bit 7 of byte j is set
+// iff r_j >= d, i.e. iff WA j has NO line flag; the same with r mod 32 and
+// d_s <= 32 for sectors.  Byte j of quad q of a group is WA 4q + j; its flag
+// is moved to bit 8j + q of the group mask (shift by 7 - q, mask
+// 0x01010101 << q), so the per-group classification of hot_row applies
+// unchanged.  9 lane ops per quad: 2.25 per WA and lane.
+// Pipe balance: the adds and the right shifts run on the FMA pipe (IMAD with
+// a runtime `one`, IMAD.HI by 2^(25+q)), the masks on the ALU pipe (LOP3):
+// 5 FMA + 4 ALU ops per quad instead of 9 ALU ops.
+__device__ __forceinline__ uint32_t add_fma(uint32_t a, uint32_t b, uint32_t one) {
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(one), "r"(b));
+    return d;
+}
+
+__device__ __forceinline__ void swar_quad(uint32_t R, uint32_t KL, uint32_t KS, uint32_t q, uint32_t valid,
+                                          uint32_t one, uint32_t& m, uint32_t& ms) {
+    const uint32_t T = add_fma(R, KL, one);                 // bit 7 of byte j: no line flag
+    const uint32_t Ts = add_fma(R & 0x1F1F1F1Fu, KS, one);  // bit 7 of byte j: no sector flag
+    const uint32_t sel = (0x01010101u << q) & valid;
+    const uint32_t x = q == 7 ? T : __umulhi(T, 1u << (25 + q));      // T >> (7 - q)
+    const uint32_t xs = q == 7 ? Ts : __umulhi(Ts, 1u << (25 + q));
+    m |= ~x & sel;
+    ms |= ~xs & sel;
+}
+
+template <int TC>
+__device__ __forceinline__ void hot_row_swar(uint32_t r0, uint32_t cr, uint32_t KL, uint32_t KS, uint32_t len,
+                                             uint32_t one, Acc& a) {
+    const uint32_t S4 = ((4u * cr) & 127u) * 0x01010101u;  // per-byte residue step of 4 WAs
+    // bytes r0 + j*cr (mod 128), j = 0..3
+    uint32_t R = (r0 & 127u) | (((r0 + cr) & 127u) << 8) | (((r0 + 2u * cr) & 127u) << 16) |
+                 (((r0 + 3u * cr) & 127u) << 24);
+    uint32_t sf = 0;
+    while (len >= 32) {                                     // full groups: shifts are immediates
+        uint32_t m = 0, ms = 0;
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            swar_quad(R, KL, KS, uint32_t(q), 0xffffffffu, one, m, ms);
+            R = add_fma(R, S4, one) & 0x7F7F7F7Fu;
+        }
+        group_end<TC>(m, 32, a);
+        sf += __popc(ms);
+        len -= 32;
+    }
+    if (len) {                                              // partial group
+        uint32_t m = 0, ms = 0, q = 0;
+        for (uint32_t i = 0; i < len; i += 4, q++) {
+            const uint32_t k = len - i;                     // WAs left; bytes >= k are past the row
+            const uint32_t valid = k >= 4 ? 0xffffffffu : (1u << (8 * k)) - 1u;
+            swar_quad(R, KL, KS, q, valid, one, m, ms);
+            R = add_fma(R, S4, one) & 0x7F7F7F7Fu;
+        }
+        group_end<TC>(m, len, a);
+        sf += __popc(ms);
+    }
+    a.sf += sf;
+}
+
 // MATCH: literal __match_any_sync expansion over 64-bit lane addresses.
 __device__ __forceinline__ void hot_match(int64_t addr, int64_t step, uint32_t len, uint32_t tmin, Acc& a) {
     const unsigned lt = lanemask_lt();
@@ -276,9 +340,11 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
 // ------------------------------------------------------------- per access
 // Count WAs [off, off + cnt) of access `a` (instance order: warp-rep, then
 // inner tuple with the last inner loop fastest).  DEPTH = a.depth.
-template <bool MATCH, int DEPTH, int TC>
+// MODE: 0 = MATCH (__match_any_sync), 1 = scalar residue, 2 = byte-sliced residue.
+template <int MODE, int DEPTH, int TC>
 __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B, uint64_t T0,
-                             uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t cnt, int lane, Acc& acc) {
+                             uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t cnt, int lane, uint32_t one,
+                             Acc& acc) {
     const uint32_t tmin = (32u * a.elem_bytes + 127u) / 128u;       // R11
     const uint64_t Tl = DEPTH == 1 ? T0 : DEPTH == 2 ? T1 : DEPTH == 3 ? T2 : 1;
     const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
@@ -293,9 +359,9 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     warp_seek(it, m, P, B);
     while (cnt > 0) {
         const int64_t A = lane_address(nest, a, it, lane);
-        uint32_t u_low = 0, dl = 0, ds = 0;
+        uint32_t u_low = 0, dl = 0, ds = 0, KL = 0, KS = 0;
         int64_t Am = A;
-        if (!MATCH) {
+        if (MODE != 0) {
             int64_t upper;
             uint64_t gap;
             if (nest.par_dims == 1) {
@@ -312,6 +378,11 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
             u_low = uint32_t(upper);
             dl = has ? (gap >= 128 ? 0xffffffffu : uint32_t(gap) << 25) : 0u;
             ds = has ? (gap >= 32 ? 0xffffffffu : uint32_t(gap) << 27) : 0u;
+            // byte-sliced thresholds: d capped at 128 (lines) / 32 (sectors); 0 = never a flag
+            const uint32_t dlb = has ? uint32_t(umin64(gap, 128)) : 0u;
+            const uint32_t dsb = has ? uint32_t(umin64(gap, 32)) : 0u;
+            KL = 0x80808080u - dlb * 0x01010101u;
+            KS = 0x80808080u - dsb * 0x01010101u;
         } else {
             const int64_t a0 = __shfl_sync(kFull, A, 0);
             Am = lane < int(it.n) ? A : a0;         // inactive lanes duplicate lane 0
@@ -326,13 +397,16 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
             if (DEPTH >= 3) D += a.c_inner[2] * int64_t(i2);
             const uint64_t il = DEPTH == 1 ? i0 : DEPTH == 2 ? i1 : DEPTH == 3 ? i2 : 0;
             const uint32_t len = uint32_t(umin64(Tl - il, left));
-            if (MATCH) {
+            if (MODE == 0) {
                 hot_match(Am + D, cl, len, tmin, acc);
-            } else {
+            } else if (TC == 4 || MODE == 1) {
                 const uint32_t y = (u_low + uint32_t(uint64_t(D))) << 25;
                 const uint32_t step = uint32_t(uint64_t(cl)) << 25;
                 if (TC == 4) hot_row_t4(y, step, dl, ds, len, acc);
-                else hot_row<TC>(y, step, dl, ds, len, acc);
+                else hot_row<TC == 4 ? 1 : TC>(y, step, dl, ds, len, acc);
+            } else {
+                hot_row_swar<TC == 4 ? 1 : TC>(u_low + uint32_t(uint64_t(D)), uint32_t(uint64_t(cl)) & 127u, KL,
+                                               KS, len, one, acc);
             }
             left -= len;
             // odometer carry (registers only)
@@ -365,7 +439,7 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
     acc = Acc{};
 }
 
-template <bool MATCH>
+template <int MODE>
 __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane) {
     const sel_nest nest = a.nests[a.prob_nest[q]];
     const uint32_t B = a.prob_B[q];
@@ -386,19 +460,19 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
         const int tc = (32 * int(ac.elem_bytes) + 127) / 128;     // tmin (R11): 1, 2 or 4
 #define SEL_DISPATCH(M, TCV)                                                                          \
     switch (d) {                                                                                      \
-    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
-    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
-    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;        \
-    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, acc); break;       \
+    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
+    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
+    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
+    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;       \
     }
-        if (MATCH) {
-            SEL_DISPATCH(true, 1)
+        if (MODE == 0) {
+            SEL_DISPATCH(0, 1)
         } else if (tc == 1) {
-            SEL_DISPATCH(false, 1)
+            SEL_DISPATCH(MODE, 1)
         } else if (tc == 2) {
-            SEL_DISPATCH(false, 2)
+            SEL_DISPATCH(MODE, 2)
         } else {
-            SEL_DISPATCH(false, 4)
+            SEL_DISPATCH(MODE, 4)
         }
 #undef SEL_DISPATCH
         take -= t;
@@ -407,13 +481,13 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
     flush(a, q, acc, lane);
 }
 
-template <bool MATCH>
 #ifndef SEL_COUNT_MIN_BLOCKS
 #define SEL_COUNT_MIN_BLOCKS 3
 #endif
 #ifndef SEL_COUNT_THREADS
 #define SEL_COUNT_THREADS 256
 #endif
+template <int MODE>
 __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t nq = a.hdr->n_problems;
@@ -440,7 +514,7 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
                 continue;
             }
             const uint32_t take = uint32_t(umin64(Wq - off, len));
-            count_problem<MATCH>(a, q, off, take, lane);
+            count_problem<MODE>(a, q, off, take, lane);
             len -= take;
             off = 0;
             q++;
@@ -448,24 +522,28 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
     }
 }
 
-cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_problems, uint32_t flags,
-                         cudaStream_t s) {
-    (void)max_problems;
-    static int grid[2] = {0, 0};
-    const bool match = (flags & SEL_F_MATCH_ANY) != 0;
-    int& g = grid[match ? 1 : 0];
+template <int MODE>
+static int count_grid() {
+    static int g = 0;
     if (g == 0) {
         int dev = 0, sms = 0, per = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (match) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<true>, SEL_COUNT_THREADS, 0);
-        else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<false>, SEL_COUNT_THREADS, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<MODE>, SEL_COUNT_THREADS, 0);
         g = sms * (per > 0 ? per : 1);
     }
-    CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr};
+    return g;
+}
+
+cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_problems, uint32_t flags,
+                         cudaStream_t s) {
+    (void)max_problems;
+    const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
+    CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u};
     prof_before_count(s);
-    if (match) k_count<true><<<g, SEL_COUNT_THREADS, 0, s>>>(a);
-    else k_count<false><<<g, SEL_COUNT_THREADS, 0, s>>>(a);
+    if (mode == 0) k_count<0><<<count_grid<0>(), SEL_COUNT_THREADS, 0, s>>>(a);
+    else if (mode == 1) k_count<1><<<count_grid<1>(), SEL_COUNT_THREADS, 0, s>>>(a);
+    else k_count<2><<<count_grid<2>(), SEL_COUNT_THREADS, 0, s>>>(a);
     prof_after_count(s);
     note_launch();
     return cudaGetLastError();

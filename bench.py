@@ -116,13 +116,28 @@ def measured_peaks():
         return {}
 
 
-def ncu_traffic_per_launch():
-    """dram bytes per counting-kernel launch from the committed ncu capture."""
+def ncu_capture():
+    """Counters of the committed ncu --set full capture of the counting kernel
+    in this bench configuration (profiles/ncu_count_kernel.json)."""
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_count_kernel.json")) as f:
-            return json.load(f).get("dram_bytes_per_launch")
+            d = json.load(f)
     except (OSError, ValueError):
-        return None
+        return {}
+    k = d.get("count_kernel_full", {})
+    out = {"traffic": d.get("dram_bytes_per_launch"),
+           "warp_instructions_per_wa": d.get("warp_instructions_per_wa")}
+    for key, name in (("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "alu_pipe_pct"),
+                      ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "fma_pipe_pct"),
+                      ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue_active_pct")):
+        if key in k:
+            out[name] = k[key]
+    return out
+
+
+def ncu_traffic_per_launch():
+    """dram bytes per counting-kernel launch from the committed ncu capture."""
+    return ncu_capture().get("traffic")
 
 
 def cpu_oracle_sample(batch, seconds: float, total_candidates: int):
@@ -295,13 +310,19 @@ def run_ours(args):
                                "ALU and FMA pipes both issuing) at the run's clocks",
                 "peak_alu_pipe_only": int_peak["alu"] / 1e12, "peak_fma_pipe_only": int_peak["fma"] / 1e12,
                 "peak_nominal_issue": 148 * 128 * f_mhz * 1e6 / 1e12,
-                "algorithmic_ops_per_wa": OPS_PER_WA}
+                "algorithmic_ops_per_wa": OPS_PER_WA,
+                "note": ("achieved counts SURVEY's 224 integer lane-ops per warp-access; the default "
+                         "byte-sliced primitive evaluates 4 warp-accesses per 32-bit lane op, so achieved "
+                         "can exceed the INT32 lane-op peak (frac > 1) while the pipes are not saturated; "
+                         "ncu_* are the issued-instruction counters of the committed capture"),
+                "ncu": ncu_capture()}
     hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
     line = {"metric": METRIC, "value": total / t_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_step * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
             "config": {"workload": WORKLOAD, "candidates": total, "count_sharing": not (args.flags & 1),
-                       "counting_primitive": "match_any" if args.flags & 2 else "residue",
+                       "counting_primitive": ("match_any" if args.flags & 2 else
+                                              "residue (scalar)" if args.flags & 4 else "residue (byte-sliced)"),
                        "l2": "inputs larger than L2 (2.4 GB of candidates per pass)",
                        "parallelism": f"dp{world} (candidate shards) + NCCL all-gather of decisions"},
             "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,

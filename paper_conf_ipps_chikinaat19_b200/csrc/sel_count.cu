@@ -222,13 +222,31 @@ __device__ __forceinline__ uint32_t add_fma(uint32_t a, uint32_t b, uint32_t one
     return d;
 }
 
+#ifndef SEL_SWAR_FMA_ADD
+#define SEL_SWAR_FMA_ADD 0
+#endif
+#ifndef SEL_SWAR_FMA_SHIFT
+#define SEL_SWAR_FMA_SHIFT 0
+#endif
+__device__ __forceinline__ uint32_t swar_add(uint32_t a, uint32_t b, uint32_t one) {
+    if (SEL_SWAR_FMA_ADD) return add_fma(a, b, one);
+    (void)one;
+    return a + b;
+}
+
 __device__ __forceinline__ void swar_quad(uint32_t R, uint32_t KL, uint32_t KS, uint32_t q, uint32_t valid,
                                           uint32_t one, uint32_t& m, uint32_t& ms) {
-    const uint32_t T = add_fma(R, KL, one);                 // bit 7 of byte j: no line flag
-    const uint32_t Ts = add_fma(R & 0x1F1F1F1Fu, KS, one);  // bit 7 of byte j: no sector flag
+    const uint32_t T = swar_add(R, KL, one);                 // bit 7 of byte j: no line flag
+    const uint32_t Ts = swar_add(R & 0x1F1F1F1Fu, KS, one);  // bit 7 of byte j: no sector flag
     const uint32_t sel = (0x01010101u << q) & valid;
-    const uint32_t x = q == 7 ? T : __umulhi(T, 1u << (25 + q));      // T >> (7 - q)
-    const uint32_t xs = q == 7 ? Ts : __umulhi(Ts, 1u << (25 + q));
+    uint32_t x, xs;                                          // T >> (7 - q)
+    if (SEL_SWAR_FMA_SHIFT && q != 7) {
+        x = __umulhi(T, 1u << (25 + q));
+        xs = __umulhi(Ts, 1u << (25 + q));
+    } else {
+        x = T >> (7 - q);
+        xs = Ts >> (7 - q);
+    }
     m |= ~x & sel;
     ms |= ~xs & sel;
 }
@@ -241,12 +259,27 @@ __device__ __forceinline__ void hot_row_swar(uint32_t r0, uint32_t cr, uint32_t 
     uint32_t R = (r0 & 127u) | (((r0 + cr) & 127u) << 8) | (((r0 + 2u * cr) & 127u) << 16) |
                  (((r0 + 3u * cr) & 127u) << 24);
     uint32_t sf = 0;
+#ifndef SEL_SWAR_CHAINS
+#define SEL_SWAR_CHAINS 1
+#endif
+    const uint32_t S8 = ((8u * cr) & 127u) * 0x01010101u;
     while (len >= 32) {                                     // full groups: shifts are immediates
         uint32_t m = 0, ms = 0;
+        if (SEL_SWAR_CHAINS == 2) {                         // two independent residue chains (ILP)
+            uint32_t Rb = swar_add(R, S4, one) & 0x7F7F7F7Fu;
 #pragma unroll
-        for (int q = 0; q < 8; q++) {
-            swar_quad(R, KL, KS, uint32_t(q), 0xffffffffu, one, m, ms);
-            R = add_fma(R, S4, one) & 0x7F7F7F7Fu;
+            for (int q = 0; q < 8; q += 2) {
+                swar_quad(R, KL, KS, uint32_t(q), 0xffffffffu, one, m, ms);
+                swar_quad(Rb, KL, KS, uint32_t(q + 1), 0xffffffffu, one, m, ms);
+                R = swar_add(R, S8, one) & 0x7F7F7F7Fu;
+                Rb = swar_add(Rb, S8, one) & 0x7F7F7F7Fu;
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                swar_quad(R, KL, KS, uint32_t(q), 0xffffffffu, one, m, ms);
+                R = swar_add(R, S4, one) & 0x7F7F7F7Fu;
+            }
         }
         group_end<TC>(m, 32, a);
         sf += __popc(ms);
@@ -258,7 +291,7 @@ __device__ __forceinline__ void hot_row_swar(uint32_t r0, uint32_t cr, uint32_t 
             const uint32_t k = len - i;                     // WAs left; bytes >= k are past the row
             const uint32_t valid = k >= 4 ? 0xffffffffu : (1u << (8 * k)) - 1u;
             swar_quad(R, KL, KS, q, valid, one, m, ms);
-            R = add_fma(R, S4, one) & 0x7F7F7F7Fu;
+            R = swar_add(R, S4, one) & 0x7F7F7F7Fu;
         }
         group_end<TC>(m, len, a);
         sf += __popc(ms);

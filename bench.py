@@ -41,7 +41,8 @@ def parse():
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", type=int, default=5)
+    p.add_argument("--config", type=int, default=5,
+                   help="BASELINE config 1..5 (5 = the metric's workload; 4 = warp-range split across ranks)")
     p.add_argument("--candidates", type=int, default=0, help="override the batch size (testing)")
     p.add_argument("--flags", type=int, default=0, help="libsel flags (1 no count sharing, 2 match_any)")
     p.add_argument("--no-e2e", action="store_true")
@@ -218,7 +219,10 @@ def run_ours(args):
     rank, world, local = D.init()
     dev = torch.device("cuda", local)
     total = gen.num_candidates(args.config) if not args.candidates else args.candidates
-    c0, c1 = D.shard_range(total, rank, world)
+    # config 4 (192 huge candidates) splits every candidate's warp-accesses across ranks
+    # (SURVEY §8(e)); the others shard candidates by index range
+    split = args.config == 4 and world > 1
+    c0, c1 = (0, total) if split else D.shard_range(total, rank, world)
     t_gen = time.perf_counter()
     batch = gen.generate(args.config, c0, c1)
     t_gen = time.perf_counter() - t_gen
@@ -232,9 +236,12 @@ def run_ours(args):
 
     def step():
         nonlocal out
-        out = ev.evaluate(cands, out=out)
-        if world > 1:
-            D.gather_decisions(out["decision"], total, world, out=gathered)
+        if split:
+            out = D.evaluate_split(cands, ev.tables, ev.workspace, rank, world, args.flags)
+        else:
+            out = ev.evaluate(cands, out=out)
+            if world > 1:
+                D.gather_decisions(out["decision"], total, world, out=gathered)
 
     int_peak = {"alu": sel.int_peak(0), "fma": sel.int_peak(1), "both": sel.int_peak(2)}
     for _ in range(args.warmup):
@@ -267,7 +274,7 @@ def run_ours(args):
 
     # ---- end to end through the public API: pinned host inputs -> decisions + cycles on the host
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not split:
         # every step uploads its inputs (candidates + nest and access tables) from pinned host
         # memory and downloads decision + cycles to pinned host memory; sel.HostPipeline overlaps
         # step k+1's upload and step k-1's download with step k's kernels (two device slots)
@@ -304,7 +311,7 @@ def run_ours(args):
     achieved = wa_per_launch * OPS_PER_WA / (avg_count_ms / 1e3)
     roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
                 "frac": achieved / peak_ops, "traffic": ncu_traffic_per_launch(),
-                "kernel": "sel::k_count<false>", "count_ms_per_launch": avg_count_ms,
+                "kernel": "sel::k_count<%d>" % (0 if args.flags & 2 else 1 if args.flags & 4 else 2), "count_ms_per_launch": avg_count_ms,
                 "count_share_of_step": avg_count_ms / (t_step * 1e3),
                 "peak_source": "measured: sel_int_peak (independent IADD3/LOP3 + IMAD chains, all SMs, "
                                "ALU and FMA pipes both issuing) at the run's clocks",
@@ -317,14 +324,18 @@ def run_ours(args):
                          "ncu_* are the issued-instruction counters of the committed capture"),
                 "ncu": ncu_capture()}
     hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
+    workload = WORKLOAD if args.config == 5 else f"c{args.config}: BASELINE.json configs[{args.config - 1}]"
+    parallelism = (f"dp{world} (warp-range split of every candidate) + all_reduce(SUM) of u64 counters" if split
+                   else f"dp{world} (candidate shards) + NCCL all-gather of decisions")
     line = {"metric": METRIC, "value": total / t_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_step * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
-            "config": {"workload": WORKLOAD, "candidates": total, "count_sharing": not (args.flags & 1),
+            "config": {"workload": workload, "candidates": total, "count_sharing": not (args.flags & 1),
                        "counting_primitive": ("match_any" if args.flags & 2 else
                                               "residue (scalar)" if args.flags & 4 else "residue (byte-sliced)"),
-                       "l2": "inputs larger than L2 (2.4 GB of candidates per pass)",
-                       "parallelism": f"dp{world} (candidate shards) + NCCL all-gather of decisions"},
+                       "l2": (f"inputs larger than L2 ({24 * total / 1e9:.1f} GB of candidates per pass)"
+                              if 24 * total > 126e6 else "inputs fit in L2 (not the metric workload)"),
+                       "parallelism": parallelism},
             "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
             "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
             "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,

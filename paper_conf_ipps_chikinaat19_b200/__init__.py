@@ -105,16 +105,21 @@ class DeviceTables:
 
 
 def count_transactions(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor, flags: int = 0,
-                       out=None, status=None, stream=None):
-    """sel_count_transactions -> (counts int64[n, 6], status uint8[n])."""
+                       out=None, status=None, stream=None, part: int = 0, n_parts: int = 1):
+    """sel_count_transactions (or sel_count_transactions_part when n_parts > 1)
+    -> (counts int64[n, 6], status uint8[n])."""
     _require_cuda(cands, workspace)
     n = _n(cands, "candidate")
     dev = cands.device
     out = torch.empty((n, 6), dtype=torch.int64, device=dev) if out is None else out
     status = torch.empty(n, dtype=torch.uint8, device=dev) if status is None else status
     wp, wb = _ws_ptr(workspace)
-    _lib.check(_lib.lib().sel_count_transactions(_ptr(cands), n, tables.ref(), _ptr(out), _ptr(status), wp, wb,
-                                                 flags, _stream(stream)))
+    if n_parts == 1 and part == 0:
+        _lib.check(_lib.lib().sel_count_transactions(_ptr(cands), n, tables.ref(), _ptr(out), _ptr(status), wp, wb,
+                                                     flags, _stream(stream)))
+    else:
+        _lib.check(_lib.lib().sel_count_transactions_part(_ptr(cands), n, tables.ref(), part, n_parts, _ptr(out),
+                                                          _ptr(status), wp, wb, flags, _stream(stream)))
     return out, status
 
 

@@ -95,6 +95,7 @@ def lib():
         L.sel_workspace_size.restype = sz
         L.sel_workspace_size.argtypes = [u64, u64, u32]
         L.sel_count_transactions.argtypes = [vp, u64, T, vp, vp, vp, sz, u32, vp]
+        L.sel_count_transactions_part.argtypes = [vp, u64, T, u32, u32, vp, vp, vp, sz, u32, vp]
         L.sel_predict_gpu_cycles.argtypes = [vp, u64, T, vp, vp, vp, vp, vp]
         L.sel_select.argtypes = [vp, u64, vp, vp, vp, vp]
         L.sel_evaluate.argtypes = [vp, u64, T, vp, vp, vp, vp, vp, vp, sz, u32, vp]
@@ -124,7 +125,7 @@ def check(rc: int):
         raise SelError(rc, lib().sel_last_error().decode(errors="replace"))
 
 
-EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions",
+EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions", "sel_count_transactions_part",
             "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_select_launch", "sel_model_cpu_cost", "sel_bind_accesses", "sel_read_stats",
             "sel_profile_enable", "sel_profile_read", "sel_kernel_launches", "sel_int_peak", "sel_last_error",
             "sel_version", "sel_sizeof", "sel_offsetof")

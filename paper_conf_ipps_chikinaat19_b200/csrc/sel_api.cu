@@ -102,8 +102,8 @@ static int check_ws(void* ws, size_t bytes, uint64_t n, uint64_t n_nests, uint32
 }
 
 static int plan_and_count(const sel_candidate* c, uint64_t n, const sel_tables* t, const WsPtrs& w, uint32_t flags,
-                          cudaStream_t s) {
-    cudaError_t e = launch_plan(c, n, *t, n_device_sets(), w, t->n_nests, flags, s);
+                          cudaStream_t s, uint32_t part = 0, uint32_t n_parts = 1) {
+    cudaError_t e = launch_plan(c, n, *t, n_device_sets(), w, t->n_nests, flags, part, n_parts, s);
     if (e != cudaSuccess) return cuda_fail(e, "plan");
     e = launch_count(*t, w, n, flags, s);
     if (e != cudaSuccess) return cuda_fail(e, "count");
@@ -139,13 +139,20 @@ size_t sel_workspace_size(uint64_t n, uint64_t n_nests, uint32_t flags) {
 
 int sel_count_transactions(const sel_candidate* c, uint64_t n, const sel_tables* t, sel_counts* out,
                            uint8_t* status, void* ws, size_t ws_bytes, uint32_t flags, sel_stream_t stream) {
+    return sel_count_transactions_part(c, n, t, 0, 1, out, status, ws, ws_bytes, flags, stream);
+}
+
+int sel_count_transactions_part(const sel_candidate* c, uint64_t n, const sel_tables* t, uint32_t part,
+                                uint32_t n_parts, sel_counts* out, uint8_t* status, void* ws, size_t ws_bytes,
+                                uint32_t flags, sel_stream_t stream) {
+    if (n_parts < 1 || part >= n_parts) return fail(SEL_EINVAL, "need 0 <= part < n_parts%s");
     if (int r = check_common(c, n, t)) return r;
     if (n == 0) return SEL_OK;
     if (!out || !status) return fail(SEL_EINVAL, "out/status is NULL%s");
     if (int r = check_ws(ws, ws_bytes, n, t->n_nests, flags)) return r;
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     const WsPtrs w = ws_ptrs(ws, n, t->n_nests, flags);
-    if (int r = plan_and_count(c, n, t, w, flags, s)) return r;
+    if (int r = plan_and_count(c, n, t, w, flags, s, part, n_parts)) return r;
     cudaError_t e = launch_gather_counts(n, w, out, status, s);
     if (e != cudaSuccess) return cuda_fail(e, "gather");
     return SEL_OK;

@@ -525,8 +525,9 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
     const int lane = threadIdx.x & 31;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;
-    const uint64_t total = a.prefix[nq];
-    if (total == 0) return;
+    const uint64_t base = a.hdr->w_begin, end = a.hdr->w_end;   // this call's slice of [0, prefix[nq])
+    if (end <= base) return;
+    const uint64_t total = end - base;
     const uint64_t nwarps = uint64_t(gridDim.x) * (blockDim.x >> 5);
     uint64_t ch = total / (nwarps * 16);
     ch = ch < 256 ? 256 : (ch > kMaxChunk ? kMaxChunk : ch);
@@ -534,9 +535,9 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
         unsigned long long chunk = 0;
         if (lane == 0) chunk = atomicAdd(&a.hdr->chunk_ctr, 1ull);
         chunk = __shfl_sync(kFull, chunk, 0);
-        const uint64_t start = chunk * ch;
-        if (start >= total) break;
-        uint32_t len = uint32_t(umin64(ch, total - start));
+        if (chunk * ch >= total) break;
+        const uint64_t start = base + chunk * ch;
+        uint32_t len = uint32_t(umin64(ch, end - start));
         uint64_t q = find_problem(a.prefix, nq, start, lane);
         uint64_t off = start - a.prefix[q];
         while (len > 0) {

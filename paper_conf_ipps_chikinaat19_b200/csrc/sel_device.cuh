@@ -25,7 +25,9 @@ struct WsHeader {
     unsigned long long chunk_ctr;      // dynamic work counter of the count kernel
     unsigned int n_overflow;           // problems allocated past the slot table
     unsigned int _pad0;
-    unsigned long long _pad[21];
+    unsigned long long w_begin, w_end; // this call's slice of the problem work space (prefix units)
+    unsigned int part, n_parts;        // sel_count_transactions_part: slice index / count
+    unsigned long long _pad[18];
 };
 static_assert(sizeof(WsHeader) == 256, "header size");
 

@@ -34,7 +34,8 @@ void prof_after_count(cudaStream_t s);
 
 // sel_plan.cu: candidates -> counting problems, closed-form W per problem, prefix
 cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables& t, int n_sets,
-                        const WsPtrs& w, uint64_t n_nests, uint32_t flags, cudaStream_t s);
+                        const WsPtrs& w, uint64_t n_nests, uint32_t flags, uint32_t part, uint32_t n_parts,
+                        cudaStream_t s);
 // sel_count.cu: the hot kernel
 cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_problems, uint32_t flags,
                          cudaStream_t s);

@@ -206,9 +206,11 @@ __global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict_
 }
 
 __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_base, uint64_t n_nests,
-                                uint64_t n, int dedup) {
+                                uint64_t n, int dedup, uint32_t part, uint32_t n_parts) {
     unsigned long long np = dedup ? nest_base[n_nests] + hdr->n_overflow : n;
     hdr->n_problems = np;
+    hdr->part = part;
+    hdr->n_parts = n_parts;
     hdr->chunk_ctr = 0;
     hdr->stats.n_candidates = n;
     hdr->stats.n_problems = np;
@@ -236,12 +238,20 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader*
     prob_W[q] = WR * M_it;
 }
 
+// slice [total*part/n_parts, total*(part+1)/n_parts) of the problem work space
+// (one huge candidate's warp-accesses split R ways)
 __global__ void k_plan_stats(WsHeader* hdr, const unsigned long long* prefix) {
-    hdr->stats.wa_analysed = prefix[hdr->n_problems];
+    const unsigned __int128 total = prefix[hdr->n_problems];
+    const uint64_t b = uint64_t(total * hdr->part / hdr->n_parts);
+    const uint64_t e = uint64_t(total * (hdr->part + 1) / hdr->n_parts);
+    hdr->w_begin = b;
+    hdr->w_end = e;
+    hdr->stats.wa_analysed = e - b;
 }
 
 cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables& t, int n_sets,
-                        const WsPtrs& w, uint64_t n_nests, uint32_t flags, cudaStream_t s) {
+                        const WsPtrs& w, uint64_t n_nests, uint32_t flags, uint32_t part, uint32_t n_parts,
+                        cudaStream_t s) {
     const bool dedup = !(flags & SEL_F_NO_DEDUP);
     cudaError_t e = cudaMemsetAsync(w.hdr, 0, sizeof(WsHeader), s);
     if (e != cudaSuccess) return e;
@@ -264,7 +274,7 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
                                                            w.hdr);
         note_launch();
     }
-    k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0);
+    k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0, part, n_parts);
     k_problem_w<<<unsigned((n + 255) / 256), 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
                                                           w.prob_status, w.prob_cnt);
     note_launch(2);

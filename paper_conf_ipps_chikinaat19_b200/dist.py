@@ -5,7 +5,8 @@ range of the candidate index space with no data-path exchange; the only
 collective is the all-gather of the per-candidate decisions the north star
 asks for (NCCL over NVLink / NVSwitch on a GPU box, gloo in the CPU tests).
 Ranges are padded to a common length so a single ``all_gather_into_tensor``
-suffices; padding bytes are dropped after the gather.
+suffices; padding bytes are dropped after the gather.  Config 4 (a few huge
+candidates) splits each candidate's warp-accesses instead (``evaluate_split``).
 """
 from __future__ import annotations
 
@@ -88,6 +89,33 @@ def gather_decisions(local: torch.Tensor, total: int, world: int, out: torch.Ten
         c0, c1 = shard_range(total, r, world)
         parts.append(full[r * n_pad: r * n_pad + (c1 - c0)])
     return torch.cat(parts)
+
+
+def all_reduce_sum_(t: torch.Tensor, world: int, group=None) -> torch.Tensor:
+    """In-place element-wise SUM over ranks (exact for integer tensors)."""
+    if world == 1:
+        return t
+    if _host_staged(t):
+        h = t.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def evaluate_split(cands: torch.Tensor, tables, workspace: torch.Tensor, rank: int, world: int, flags: int = 0,
+                   group=None) -> dict:
+    """a few huge candidates, so every rank takes ALL
+    candidates but only its 1/world slice of their warp-accesses
+    (``sel_count_transactions_part``); one ``all_reduce(SUM)`` of the u64
+    counters makes them exact and every rank then runs a4-a7 identically."""
+    from . import count_transactions, predict_gpu_cycles, select
+    counts, status = count_transactions(cands, tables, workspace, flags, part=rank, n_parts=world)
+    all_reduce_sum_(counts, world, group)
+    cycles, t_gpu = predict_gpu_cycles(cands, tables, counts, status)
+    decision = select(cands, t_gpu, status)
+    return dict(counts=counts, status=status, cycles=cycles, t_gpu=t_gpu, decision=decision)
 
 
 def max_over_ranks(x: float, world: int, device) -> float:

@@ -45,7 +45,10 @@ def _worker(rank, world, port, total, q):
     full = D.gather_decisions(local, total, w)
     t = D.max_over_ranks(float(rank + 1), w, torch.device("cpu"))
     s = D.sum_over_ranks(c1 - c0, w, torch.device("cpu"))
-    q.put((rank, full.numpy().tobytes(), t, s))
+    # config-4 partial counters: parts near 2^62 sum exactly (int64, no float staging)
+    part = torch.tensor([[(1 << 62) - 7 + rank, rank, 3 * rank + 1]], dtype=torch.int64)
+    red = D.all_reduce_sum_(part, w).tolist()
+    q.put((rank, full.numpy().tobytes(), t, s, red))
     dist.destroy_process_group()
 
 
@@ -67,6 +70,7 @@ def test_gather_decisions_two_ranks_gloo(total):
     nests_global = np.concatenate([gen.generate(5, *D.shard_range(total, r, 2)).cands["nest_id"] for r in range(2)])
     devs = b.cands["device_id"]
     expect = ((nests_global + devs) % 3).astype(np.uint8)
-    for rank, full, t, s in res:
+    for rank, full, t, s, red in res:
         assert np.frombuffer(full, np.uint8).tolist() == expect.tolist()
         assert t == 2.0 and s == total
+        assert red == [[2 * ((1 << 62) - 7) + 1, 1, 5]]

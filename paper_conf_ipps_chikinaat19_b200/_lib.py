@@ -17,6 +17,7 @@ SEL_OK, SEL_EINVAL, SEL_ERANGE, SEL_ELAUNCH, SEL_ENODEV, SEL_ECUDA, SEL_EINTERNA
 SEL_F_NO_DEDUP = 1
 SEL_F_MATCH_ANY = 2
 SEL_F_SCALAR = 4
+SEL_F_EXPAND_ALL = 8
 DECISION_CPU, DECISION_GPU, DECISION_INVALID = 0, 1, 0xFF
 
 
@@ -74,7 +75,8 @@ class Tables(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [("n_candidates", ctypes.c_uint64), ("n_problems", ctypes.c_uint64),
                 ("wa_analysed", ctypes.c_uint64), ("wa_covered", ctypes.c_uint64),
-                ("n_invalid", ctypes.c_uint64), ("_reserved", ctypes.c_uint64 * 3)]
+                ("n_invalid", ctypes.c_uint64), ("wa_closed_form", ctypes.c_uint64),
+                ("_reserved", ctypes.c_uint64 * 2)]
 
 
 RECORDS = (DeviceParams, Access, Nest, Launch, Candidate, Counts)

@@ -49,6 +49,7 @@ struct CountArgs {
     unsigned long long* prob_cnt;       // W, L, S, C, U per problem
     WsHeader* hdr;
     uint32_t one;                       // 1 at run time: keeps adds as IMAD on the FMA pipe
+    uint32_t closed_form;               // resolve warp-reps with uniform lane flags in closed form
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -61,6 +62,7 @@ struct CountArgs {
 struct Acc {
     uint32_t lf, sf, uf;             // per lane
     uint32_t W, C, lk, sk, uk;       // uniform
+    uint32_t K;                      // uniform: WAs resolved in closed form (statistics)
 };
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
@@ -377,7 +379,7 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
 template <int MODE, int DEPTH, int TC>
 __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t P, uint32_t B, uint64_t T0,
                              uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t cnt, int lane, uint32_t one,
-                             Acc& acc) {
+                             uint32_t closed_form, Acc& acc) {
     const uint32_t tmin = (32u * a.elem_bytes + 127u) / 128u;       // R11
     const uint64_t Tl = DEPTH == 1 ? T0 : DEPTH == 2 ? T1 : DEPTH == 3 ? T2 : 1;
     const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
@@ -392,7 +394,7 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     warp_seek(it, m, P, B);
     while (cnt > 0) {
         const int64_t A = lane_address(nest, a, it, lane);
-        uint32_t u_low = 0, dl = 0, ds = 0, KL = 0, KS = 0;
+        uint32_t u_low = 0, dl = 0, ds = 0, KL = 0, KS = 0, dlb_u = 0, dsb_u = 0;
         int64_t Am = A;
         if (MODE != 0) {
             int64_t upper;
@@ -414,6 +416,8 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
             // byte-sliced thresholds: d capped at 128 (lines) / 32 (sectors); 0 = never a flag
             const uint32_t dlb = has ? uint32_t(umin64(gap, 128)) : 0u;
             const uint32_t dsb = has ? uint32_t(umin64(gap, 32)) : 0u;
+            dlb_u = dlb;
+            dsb_u = dsb;
             KL = 0x80808080u - dlb * 0x01010101u;
             KS = 0x80808080u - dsb * 0x01010101u;
         } else {
@@ -423,6 +427,27 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
         // rows of the last inner loop within this warp-rep
         const uint64_t here64 = umin64(Mk - tt, cnt);
         uint32_t left = uint32_t(here64);
+        if (MODE != 0 && closed_form) {
+            // UNIFORM FLAGS.  A lane's line flag  (s_l + D) mod 128 < gap_l  does
+            // not depend on the inner offset D when gap_l is 0 (never) or >= 128
+            // (always); likewise sectors with 0 or >= 32.  When that holds on every
+            // lane, all WAs of this warp-rep are identical: lines = 1 + #line
+            // flags, sectors = 1 + #sector flags, coalesced <=> lines <= tmin
+            // (R11) -- added for all `left` WAs at once (exact, no expansion).
+            const bool uni = (dlb_u == 0u || dlb_u == 128u) && (dsb_u == 0u || dsb_u == 32u);
+            if (__all_sync(kFull, uni)) {
+                const uint32_t nl = __popc(__ballot_sync(kFull, dlb_u == 128u));
+                const uint32_t ns = __popc(__ballot_sync(kFull, dsb_u == 32u));
+                acc.W += left;
+                acc.K += left;
+                acc.lk += left * nl;
+                acc.sk += left * ns;
+                if (nl + 1u <= tmin) acc.C += left;
+                else acc.uk += left * nl;
+                left = 0;
+                i0 = i1 = i2 = 0;          // the warp-rep is finished (or cnt is exhausted)
+            }
+        }
         while (left > 0) {
             int64_t D = 0;
             if (DEPTH >= 1) D += a.c_inner[0] * int64_t(i0);
@@ -469,6 +494,7 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
         const uint64_t v = lane == 0 ? W : lane == 1 ? L : lane == 2 ? S : lane == 3 ? C : U;
         atomicAdd(&a.prob_cnt[q * kCntStride + lane], (unsigned long long)v);
     }
+    if (acc.K && lane == 5) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)acc.K);
     acc = Acc{};
 }
 
@@ -493,10 +519,10 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
         const int tc = (32 * int(ac.elem_bytes) + 127) / 128;     // tmin (R11): 1, 2 or 4
 #define SEL_DISPATCH(M, TCV)                                                                          \
     switch (d) {                                                                                      \
-    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
-    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
-    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;        \
-    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, acc); break;       \
+    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
+    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
+    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
+    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;       \
     }
         if (MODE == 0) {
             SEL_DISPATCH(0, 1)
@@ -573,7 +599,8 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
                          cudaStream_t s) {
     (void)max_problems;
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
-    CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u};
+    CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
+                (flags & SEL_F_EXPAND_ALL) ? 0u : 1u};
     prof_before_count(s);
     if (mode == 0) k_count<0><<<count_grid<0>(), SEL_COUNT_THREADS, 0, s>>>(a);
     else if (mode == 1) k_count<1><<<count_grid<1>(), SEL_COUNT_THREADS, 0, s>>>(a);

@@ -59,7 +59,7 @@ def assert_parity(g, ref, exact_cycles=True, ctx=""):
         assert same.all(), f"{ctx}: t_gpu not bit-exact"
 
 
-@pytest.mark.parametrize("flags", [0, 1, 2, 3, 4, 5])
+@pytest.mark.parametrize("flags", [0, 1, 2, 3, 4, 5, 8, 12])
 def test_c1_gemm(sel, flags):
     b = gen.generate(1)
     g = run_gpu(sel, b, flags)
@@ -67,7 +67,7 @@ def test_c1_gemm(sel, flags):
     assert g["counts"][0].tolist() == [24576, 532480, 532480, 8192, 524288, 2]
 
 
-@pytest.mark.parametrize("flags", [0, 2, 4])
+@pytest.mark.parametrize("flags", [0, 2, 4, 8])
 def test_c2_polybench_medium(sel, flags):
     b = gen.generate(2)
     g = run_gpu(sel, b, flags)
@@ -111,7 +111,7 @@ def test_c4_reduced_parallel_extent(sel):
     nests["P0"] = 1 << 14
     bb = gen.Batch(b.cands, nests, b.accesses, b.launches, b.devices)
     ref = oracle.evaluate(bb)
-    for flags in (0, 1, 4):
+    for flags in (0, 1, 4, 8):
         assert_parity(run_gpu(sel, bb, flags), ref, ctx=f"c4-reduced flags={flags}")
 
 
@@ -167,7 +167,7 @@ def _random_batch(seed, n):
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 1, 2, 4])
+@pytest.mark.parametrize("flags", [0, 1, 2, 4, 8, 12])
 def test_random_tiny_nests(sel, flags):
     """Random tiny nests: partial warps, B not a multiple of 32, #OMP_Rep > 1,
     collapse(2) with wrapping lanes, negative and zero strides, zero trips,
@@ -207,7 +207,7 @@ def test_invalid_and_edge_candidates(sel):
     b = gen.custom_batch(items, launches_=launches)
     ref = oracle.evaluate(b)
     assert list(ref["status"]) == [0, 1, 1, 1, 1, 1, 1, 2, 1, 1, 2, 0, 0, 0, 0, 3]
-    for flags in (0, 1, 2, 4):
+    for flags in (0, 1, 2, 4, 8):
         g = run_gpu(sel, b, flags)
         assert_parity(g, ref, ctx=f"edge flags={flags}")
         assert (g["decision"][ref["status"] != 0] == 0xFF).all()
@@ -304,7 +304,7 @@ def _random_medium_batch(seed, n):
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 2, 4])
+@pytest.mark.parametrize("flags", [0, 2, 4, 8, 12])
 def test_random_medium_nests(sel, flags):
     b = _random_medium_batch(123 + flags, 1500)
     ref = oracle.evaluate(b)
@@ -329,3 +329,51 @@ def test_count_sharing_slot_overflow(sel):
     assert_parity(g, oracle.evaluate(b), ctx="slot overflow")
     # 8 shared classes per nest; candidates of the remaining classes get private problems
     assert 3 * (8 + 6) < g["stats"]["n_problems"] <= 3 * (8 + 2 * 16)
+
+
+def _uniform_gap_batch():
+    """Lane gaps at and around the closed-form boundaries (0, 31/32/33,
+    127/128/129, negative strides), partial warps, depth 0-2 and collapse(2)
+    (per-lane gaps that are uniform on some warps and not on others)."""
+    import test_oracle_model as M
+    base = M.BASE
+    items = []
+    for cp in (0, 4, 8, 31, 32, 33, 64, 127, 128, 129, 256, 4096, -8, -128, -129, -4096):
+        for eb in (4, 8, 16):
+            for P0 in (1, 31, 33, 100):
+                if cp % eb and cp != 0:
+                    continue
+                for depth, trip, ci in ((0, [], ()), (1, [37], (eb,)), (2, [3, 45], (4096, eb)),
+                                        (1, [5], (128,)), (1, [9], (0,))):
+                    b0 = base + 8 * eb + (4096 * 200 if cp < 0 else 0)
+                    a = gen.make_access(base=b0, c_par=(cp,), c_inner=ci, elem_bytes=eb, depth=depth)
+                    items.append(dict(P0=P0, trip=trip, accesses=[a], comp=[1, 1, 1][: depth + 1]))
+    for P1, c1 in ((4, 128), (8, 8), (40, 256), (3, 0)):       # collapse(2): lane gaps c1 or row jumps
+        for c0 in (0, 512, 1 << 16):
+            a = gen.make_access(base=base, c_par=(c0, c1), c_inner=(8,), elem_bytes=8, depth=1)
+            items.append(dict(P0=70, P1=P1, par_dims=2, trip=[6], accesses=[a], comp=[1, 1]))
+    return gen.custom_batch(items)
+
+
+@pytest.mark.parametrize("flags", [0, 4, 8, 1])
+def test_uniform_flag_closed_form(sel, flags):
+    b = _uniform_gap_batch()
+    ref = oracle.evaluate(b)
+    assert (ref["status"] == 0).all()
+    g = run_gpu(sel, b, flags)
+    assert_parity(g, ref, ctx=f"uniform-gap flags={flags}")
+    st = g["stats"]
+    if flags & 8:
+        assert st["wa_closed_form"] == 0
+    else:
+        assert 0 < st["wa_closed_form"] < st["wa_analysed"]
+
+
+def test_closed_form_share_c5_slice(sel):
+    """On a c5 slice most warp-accesses have uniform lane flags (broadcast or
+    >= 128-byte lane strides); the closed form and full expansion agree."""
+    b = gen.generate(5, 0, 200000)
+    g0, g8 = run_gpu(sel, b, 0), run_gpu(sel, b, 8)
+    assert (g0["counts"] == g8["counts"]).all() and (g0["cycles"] == g8["cycles"]).all()
+    assert g0["stats"]["wa_analysed"] == g8["stats"]["wa_analysed"]
+    assert g0["stats"]["wa_closed_form"] > g0["stats"]["wa_analysed"] // 2

@@ -32,7 +32,8 @@ METRIC = "model evaluations/sec and warp-accesses analysed/sec at 1/2/4/8 B200 (
 UNIT = "evals/s"
 WORKLOAD = ("c5: 10^8-candidate selection sweep (24 Polybench-shaped nests x trip counts x "
             "8 launch configs x 4 device sets)")
-OPS_PER_WA = 224           # 7 integer lane-ops x 32 lanes per warp-access
+OPS_PER_WA = 224           # 7 integer lane-ops x 32 lanes per warp-access (lane expansion)
+OPS_PER_WA_ARITH = 12      # arithmetic-lane path, one lane per warp-access
 
 
 def parse():
@@ -307,11 +308,12 @@ def run_ours(args):
     # lane-op rate with the ALU and FMA pipes both busy (sel_int_peak mode 2), all SMs
     f_mhz = clocks["sm_mhz"] or measured_peaks().get("clocks_under_load", {}).get("sm_mhz_median", 1965.0)
     peak_ops = int_peak["both"]
-    # WAs the kernel expanded lane by lane in this rank's launch (rank 0); the rest of
-    # wa_analysed was resolved in closed form (uniform lane flags)
-    wa_per_launch = stats["wa_analysed"] - stats["wa_closed_form"]
+    # algorithmic lane-ops of this rank's launch (rank 0), per counting path (DESIGN.md §7/§8):
+    # lane-by-lane expansion 224 / WA, arithmetic lanes 12 / WA, uniform-flag closed form 0
+    wa_arith = stats["wa_arith_lanes"]
+    wa_lane = stats["wa_analysed"] - stats["wa_closed_form"] - wa_arith
     avg_count_ms = count_ms / max(count_launches, 1)
-    achieved = wa_per_launch * OPS_PER_WA / (avg_count_ms / 1e3)
+    achieved = (wa_lane * OPS_PER_WA + wa_arith * OPS_PER_WA_ARITH) / (avg_count_ms / 1e3)
     roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
                 "frac": achieved / peak_ops, "traffic": ncu_traffic_per_launch(),
                 "kernel": "sel::k_count<%d>" % (0 if args.flags & 2 else 1 if args.flags & 4 else 2), "count_ms_per_launch": avg_count_ms,
@@ -320,11 +322,14 @@ def run_ours(args):
                                "ALU and FMA pipes both issuing) at the run's clocks",
                 "peak_alu_pipe_only": int_peak["alu"] / 1e12, "peak_fma_pipe_only": int_peak["fma"] / 1e12,
                 "peak_nominal_issue": 148 * 128 * f_mhz * 1e6 / 1e12,
-                "algorithmic_ops_per_wa": OPS_PER_WA,
-                "note": ("achieved counts SURVEY's 224 integer lane-ops per EXPANDED warp-access (closed-form "
-                         "warp-reps excluded); the default "
-                         "byte-sliced primitive evaluates 4 warp-accesses per 32-bit lane op, so achieved "
-                         "can exceed the INT32 lane-op peak (frac > 1) while the pipes are not saturated; "
+                "algorithmic_ops_per_wa": {"lane_expansion": OPS_PER_WA, "arith_lanes": OPS_PER_WA_ARITH,
+                                           "closed_form": 0},
+                "wa_per_path": {"lane_expansion": wa_lane, "arith_lanes": wa_arith,
+                                "closed_form": stats["wa_closed_form"]},
+                "note": ("achieved = sum over counting paths of warp-accesses x that path's algorithmic "
+                         "lane-ops (SURVEY's 224 for lane-by-lane expansion, 12 for one lane per "
+                         "warp-access, 0 for uniform-flag closed form) / count-kernel time; the byte-sliced "
+                         "lane expansion evaluates 4 warp-accesses per 32-bit lane op; "
                          "ncu_* are the issued-instruction counters of the committed capture"),
                 "ncu": ncu_capture()}
     hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
@@ -335,7 +340,7 @@ def run_ours(args):
             "warmup": args.warmup, "ms_per_step": t_step * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
             "config": {"workload": workload, "candidates": total, "count_sharing": not (args.flags & 1),
-                       "closed_form_uniform_flags": not (args.flags & 8),
+                       "lane_pattern_paths": not (args.flags & 8),
                        "counting_primitive": ("match_any" if args.flags & 2 else
                                               "residue (scalar)" if args.flags & 4 else "residue (byte-sliced)"),
                        "l2": (f"inputs larger than L2 ({24 * total / 1e9:.1f} GB of candidates per pass)"
@@ -343,7 +348,7 @@ def run_ours(args):
                        "parallelism": parallelism},
             "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
             "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
-            "wa_closed_form_per_step": wa_closed, "wa_expanded_per_s": (wa_analysed - wa_closed) / t_step,
+            "wa_closed_form_per_step": wa_closed,
             "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
     if not args.no_next and args.config == 5:

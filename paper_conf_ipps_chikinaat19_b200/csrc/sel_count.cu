@@ -61,8 +61,9 @@ struct CountArgs {
 // MATCH paths).
 struct Acc {
     uint32_t lf, sf, uf;             // per lane
+    uint32_t cc;                     // per lane: coalesced WAs (arithmetic-lane path)
     uint32_t W, C, lk, sk, uk;       // uniform
-    uint32_t K;                      // uniform: WAs resolved in closed form (statistics)
+    uint32_t K, Q;                   // uniform statistics: WAs in closed form / arithmetic-lane path
 };
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
@@ -372,6 +373,108 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
     return a.base + a.c_par[0] * int64_t(p / nest.P1) + a.c_par[1] * int64_t(p % nest.P1);
 }
 
+// ------------------------------------------------------------- arithmetic lanes
+// A 1-D parallel access with lane stride 0 < g < 128 places the n active lanes
+// of a warp-access at lo, lo + g, ..., lo + (n-1) g (lo = the lowest lane
+// address; lanes descend when c_par < 0).  Consecutive lanes are < 128 bytes
+// apart, so no line between the first and the last is skipped:
+//   lines   = 1 + ((r + span) >> 7),  r = (lo + D) mod 128,  span = (n-1) g
+//   sectors = 1 + (((r mod 32) + span) >> 5)   if g < 32   (none skipped)
+//           = n                                  if g >= 32 (one per lane)
+// -- the same integers as the lane-by-lane definition, from one residue.  Each
+// lane therefore evaluates its OWN warp-accesses (lane l takes instances l,
+// l + 32, ... of the chunk, walking (warp-rep, inner tuple) as a mixed-radix
+// counter), 32 warp-accesses per warp instruction instead of one.
+template <int DEPTH>
+__device__ void count_arith(const sel_access& a, uint64_t P, uint32_t B, uint64_t T0, uint64_t T1, uint64_t T2,
+                            uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt, int lane, uint32_t tmin,
+                            Acc& acc) {
+    const int64_t c0 = a.c_par[0];
+    const uint32_t g = uint32_t(uabs(c0));
+    const bool neg = c0 < 0;
+    const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
+    const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
+                   k2 = uint32_t(uint64_t(a.c_inner[2]));
+    const uint32_t t0 = uint32_t(T0), t1 = uint32_t(T1), t2 = uint32_t(T2);
+    // this lane's first instance: offset tt + lane from warp-rep m0
+    const uint64_t u = tt + uint64_t(lane);
+    uint64_t m = m0 + u / Mk;
+    const uint64_t rm = u % Mk;
+    uint32_t i0 = 0, i1 = 0, i2 = 0;
+    if (DEPTH == 1) { i0 = uint32_t(rm); }
+    if (DEPTH == 2) { i1 = uint32_t(rm % T1); i0 = uint32_t(rm / T1); }
+    if (DEPTH == 3) { i2 = uint32_t(rm % T2); const uint64_t r = rm / T2; i1 = uint32_t(r % T1); i0 = uint32_t(r / T1); }
+    // the step of 32 instances as mixed-radix digits (warp-rep, i0, i1, i2)
+    const uint32_t sm = uint32_t(32 / Mk);              // 0 unless Mk < 32
+    const uint32_t sr = uint32_t(32 % Mk);
+    uint32_t d0 = 0, d1 = 0, d2 = 0;
+    if (DEPTH == 1) { d0 = sr; }
+    if (DEPTH == 2) { d1 = sr % t1; d0 = sr / t1; }
+    if (DEPTH == 3) { d2 = sr % t2; d1 = (sr / t2) % t1; d0 = (sr / t2) / t1; }
+    // warp-rep m = (block kb, warp w) when 32 does not divide B (R8, R9)
+    const bool blocked = (B & 31u) != 0;
+    const uint32_t wpb = (B + 31u) >> 5;
+    uint64_t kb = blocked ? m / wpb : 0;
+    uint32_t w = blocked ? uint32_t(m - kb * wpb) : 0u;
+    uint32_t lo32 = 0, nm1 = 0, span = 0;
+    auto warp_props = [&]() {
+        uint64_t p0, e;
+        if (blocked) {
+            p0 = kb * B + 32ull * w;
+            e = umin64(p0 + 32, (kb + 1) * uint64_t(B));
+        } else {
+            p0 = m * 32;
+            e = p0 + 32;
+        }
+        e = umin64(e, P);
+        nm1 = uint32_t(e - p0) - 1u;                   // active lanes - 1 (unused past the chunk)
+        lo32 = base32 + c032 * uint32_t(p0) + (neg ? c032 * nm1 : 0u);
+        span = nm1 * g;
+    };
+    warp_props();
+    uint32_t lf = 0, sf = 0, uf = 0, cc = 0;
+    for (uint32_t t = uint32_t(lane); t < cnt; t += 32) {
+        uint32_t D = 0;
+        if (DEPTH >= 1) D += k0 * i0;
+        if (DEPTH >= 2) D += k1 * i1;
+        if (DEPTH >= 3) D += k2 * i2;
+        const uint32_t r = (lo32 + D) & 127u;
+        const uint32_t nl = (r + span) >> 7;           // lines - 1
+        const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
+        lf += nl;
+        sf += ns;
+        if (nl + 1u <= tmin) cc++;                      // R11
+        else uf += nl;
+        uint32_t carry = 0;
+        if (DEPTH >= 3) { i2 += d2; carry = i2 >= t2; if (carry) i2 -= t2; }
+        if (DEPTH >= 2) {
+            i1 += (DEPTH == 2 ? d1 : d1 + carry);
+            carry = i1 >= t1;
+            if (carry) i1 -= t1;
+        }
+        if (DEPTH >= 1) {
+            i0 += (DEPTH == 1 ? d0 : d0 + carry);
+            carry = i0 >= t0;
+            if (carry) i0 -= t0;
+        }
+        const uint32_t dm = sm + carry;
+        if (dm) {
+            m += dm;
+            if (blocked) {
+                w += dm;
+                while (w >= wpb) { w -= wpb; kb++; }
+            }
+            warp_props();
+        }
+    }
+    acc.lf += lf;
+    acc.sf += sf;
+    acc.uf += uf;
+    acc.cc += cc;
+    acc.W += cnt;
+    acc.Q += cnt;
+}
+
 // ------------------------------------------------------------- per access
 // Count WAs [off, off + cnt) of access `a` (instance order: warp-rep, then
 // inner tuple with the last inner loop fastest).  DEPTH = a.depth.
@@ -385,6 +488,33 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
     uint64_t m = off / Mk;
     uint64_t tt = off - m * Mk;
+    if (MODE != 0 && closed_form && nest.par_dims == 1) {
+        // UNIFORM FLAGS, whole access (see below): a 1-D parallel stride g of 0 or
+        // >= 128 bytes gives every active lane after the first a line and a sector
+        // flag (g >= 128) or none (g = 0) in every warp-access, so a warp-rep with
+        // n active lanes has lines = sectors = 1 + (g ? n - 1 : 0) -- no lane work.
+        const uint64_t g = uabs(a.c_par[0]);
+        if (g == 0 || g >= 128) {
+            WarpIter it;
+            warp_seek(it, m, P, B);
+            while (cnt > 0) {
+                const uint32_t k = uint32_t(umin64(Mk - tt, cnt));
+                const uint32_t nl = g ? it.n - 1u : 0u;
+                acc.W += k;
+                acc.K += k;
+                acc.lk += k * nl;
+                acc.sk += k * nl;
+                if (nl + 1u <= tmin) acc.C += k;
+                else acc.uk += k * nl;
+                cnt -= k;
+                tt = 0;
+                if (cnt > 0) warp_next(it, P, B);
+            }
+            return;
+        }
+        count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, cnt, lane, tmin, acc);
+        return;
+    }
     // inner indices, last fastest
     uint64_t i0 = 0, i1 = 0, i2 = 0;
     if (DEPTH == 1) { i0 = tt; }
@@ -488,13 +618,14 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
     const uint64_t W = acc.W;
     const uint64_t L = W + slf + acc.lk;
     const uint64_t S = W + ssf + acc.sk;
-    const uint64_t C = acc.C;
+    const uint64_t C = acc.C + __reduce_add_sync(kFull, acc.cc);
     const uint64_t U = (W - C) + suf + acc.uk;
     if (W && lane < 5) {
         const uint64_t v = lane == 0 ? W : lane == 1 ? L : lane == 2 ? S : lane == 3 ? C : U;
         atomicAdd(&a.prob_cnt[q * kCntStride + lane], (unsigned long long)v);
     }
     if (acc.K && lane == 5) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)acc.K);
+    if (acc.Q && lane == 6) atomicAdd((unsigned long long*)&a.hdr->stats.wa_arith_lanes, (unsigned long long)acc.Q);
     acc = Acc{};
 }
 

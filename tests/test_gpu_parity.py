@@ -352,7 +352,14 @@ def _uniform_gap_batch():
         for c0 in (0, 512, 1 << 16):
             a = gen.make_access(base=base, c_par=(c0, c1), c_inner=(8,), elem_bytes=8, depth=1)
             items.append(dict(P0=70, P1=P1, par_dims=2, trip=[6], accesses=[a], comp=[1, 1]))
-    return gen.custom_batch(items)
+    # every item again under blocks whose size 32 does not divide (partial last warp
+    # of every block) and a small grid cap (#OMP_Rep > 1)
+    items += [dict(it, launch=1) for it in items] + [dict(it, launch=2) for it in items]
+    launches = np.zeros(3, gen.LAUNCH_DTYPE)
+    launches[0] = (256, 65535, 32, 0)
+    launches[1] = (48, 65535, 32, 0)
+    launches[2] = (200, 1, 32, 0)
+    return gen.custom_batch(items, launches_=launches)
 
 
 @pytest.mark.parametrize("flags", [0, 4, 8, 1])
@@ -364,9 +371,10 @@ def test_uniform_flag_closed_form(sel, flags):
     assert_parity(g, ref, ctx=f"uniform-gap flags={flags}")
     st = g["stats"]
     if flags & 8:
-        assert st["wa_closed_form"] == 0
+        assert st["wa_closed_form"] == 0 and st["wa_arith_lanes"] == 0
     else:
-        assert 0 < st["wa_closed_form"] < st["wa_analysed"]
+        assert 0 < st["wa_closed_form"] and 0 < st["wa_arith_lanes"]
+        assert st["wa_closed_form"] + st["wa_arith_lanes"] < st["wa_analysed"]     # collapse(2) expands
 
 
 def test_closed_form_share_c5_slice(sel):

@@ -373,6 +373,64 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
     return a.base + a.c_par[0] * int64_t(p / nest.P1) + a.c_par[1] * int64_t(p % nest.P1);
 }
 
+// a / b with a 32-bit fast path (the common case: both operands below 2^32)
+__device__ __forceinline__ uint64_t udiv(uint64_t a, uint64_t b) {
+    if (a < b) return 0;
+    if (((a | b) >> 32) == 0) return uint32_t(a) / uint32_t(b);
+    return a / b;
+}
+
+// ------------------------------------------------------------- uniform flags
+// A 1-D parallel stride g of 0 or >= 128 bytes gives every active lane after
+// the first a line and a sector flag (g >= 128) or none (g = 0) in every
+// warp-access, independently of the inner offset: a warp-rep with n active
+// lanes has lines = sectors = 1 + (g ? n - 1 : 0) in all of its warp-accesses.
+// Lane l adds up warp-reps m0 + l, m0 + l + 32, ... of the chunk (closed form,
+// no expansion).
+__device__ void count_uniform(uint64_t P, uint32_t B, uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt,
+                              bool flags, uint32_t tmin, int lane, Acc& acc) {
+    const uint64_t start = tt, end = tt + cnt;           // instances relative to warp-rep m0
+    const uint64_t nw = udiv(end - 1, Mk) + 1;           // warp-reps touched
+    const bool blocked = (B & 31u) != 0;
+    const uint32_t wpb = (B + 31u) >> 5;
+    uint64_t kb = 0;
+    uint32_t w = 0;
+    if (blocked) {
+        const uint64_t mm = m0 + uint64_t(lane);
+        kb = udiv(mm, wpb);
+        w = uint32_t(mm - kb * wpb);
+    }
+    const uint32_t qb = 32u / wpb, rw = 32u % wpb;       // 32 warps = qb blocks + rw warps
+    uint32_t lf = 0, cc = 0, uf = 0;
+    for (uint64_t j = uint64_t(lane); j < nw; j += 32) {
+        const uint64_t lo = j * Mk > start ? j * Mk : start;
+        const uint64_t hi = (j + 1) * Mk < end ? (j + 1) * Mk : end;
+        const uint32_t k = uint32_t(hi - lo);
+        uint64_t p0, e;
+        if (blocked) {
+            p0 = kb * B + 32ull * w;
+            e = umin64(p0 + 32, (kb + 1) * uint64_t(B));
+            kb += qb;
+            w += rw;
+            if (w >= wpb) { w -= wpb; kb++; }
+        } else {
+            p0 = (m0 + j) * 32;
+            e = p0 + 32;
+        }
+        e = umin64(e, P);
+        const uint32_t nl = flags ? uint32_t(e - p0) - 1u : 0u;
+        lf += k * nl;
+        if (nl + 1u <= tmin) cc += k;                     // R11
+        else uf += k * nl;
+    }
+    acc.lf += lf;
+    acc.sf += lf;
+    acc.cc += cc;
+    acc.uf += uf;
+    acc.W += cnt;
+    acc.K += cnt;
+}
+
 // ------------------------------------------------------------- arithmetic lanes
 // A 1-D parallel access with lane stride 0 < g < 128 places the n active lanes
 // of a warp-access at lo, lo + g, ..., lo + (n-1) g (lo = the lowest lane
@@ -398,23 +456,30 @@ __device__ void count_arith(const sel_access& a, uint64_t P, uint32_t B, uint64_
     const uint32_t t0 = uint32_t(T0), t1 = uint32_t(T1), t2 = uint32_t(T2);
     // this lane's first instance: offset tt + lane from warp-rep m0
     const uint64_t u = tt + uint64_t(lane);
-    uint64_t m = m0 + u / Mk;
-    const uint64_t rm = u % Mk;
+    const uint64_t um = udiv(u, Mk);
+    uint64_t m = m0 + um;
+    const uint64_t rm = u - um * Mk;
     uint32_t i0 = 0, i1 = 0, i2 = 0;
     if (DEPTH == 1) { i0 = uint32_t(rm); }
-    if (DEPTH == 2) { i1 = uint32_t(rm % T1); i0 = uint32_t(rm / T1); }
-    if (DEPTH == 3) { i2 = uint32_t(rm % T2); const uint64_t r = rm / T2; i1 = uint32_t(r % T1); i0 = uint32_t(r / T1); }
+    if (DEPTH == 2) { const uint64_t q = udiv(rm, T1); i0 = uint32_t(q); i1 = uint32_t(rm - q * T1); }
+    if (DEPTH == 3) {
+        const uint64_t q = udiv(rm, T2), q2 = udiv(q, T1);
+        i2 = uint32_t(rm - q * T2); i1 = uint32_t(q - q2 * T1); i0 = uint32_t(q2);
+    }
     // the step of 32 instances as mixed-radix digits (warp-rep, i0, i1, i2)
-    const uint32_t sm = uint32_t(32 / Mk);              // 0 unless Mk < 32
-    const uint32_t sr = uint32_t(32 % Mk);
+    const uint32_t sm = Mk > 32 ? 0u : 32u / uint32_t(Mk);      // 0 unless Mk <= 32
+    const uint32_t sr = Mk > 32 ? 32u : 32u % uint32_t(Mk);
     uint32_t d0 = 0, d1 = 0, d2 = 0;
     if (DEPTH == 1) { d0 = sr; }
-    if (DEPTH == 2) { d1 = sr % t1; d0 = sr / t1; }
-    if (DEPTH == 3) { d2 = sr % t2; d1 = (sr / t2) % t1; d0 = (sr / t2) / t1; }
+    if (DEPTH == 2) { d1 = sr < t1 ? sr : sr % t1; d0 = sr < t1 ? 0u : sr / t1; }
+    if (DEPTH == 3) {
+        const uint32_t q = sr < t2 ? 0u : sr / t2;
+        d2 = sr - q * t2; d1 = q < t1 ? q : q % t1; d0 = q < t1 ? 0u : q / t1;
+    }
     // warp-rep m = (block kb, warp w) when 32 does not divide B (R8, R9)
     const bool blocked = (B & 31u) != 0;
     const uint32_t wpb = (B + 31u) >> 5;
-    uint64_t kb = blocked ? m / wpb : 0;
+    uint64_t kb = blocked ? udiv(m, wpb) : 0;
     uint32_t w = blocked ? uint32_t(m - kb * wpb) : 0u;
     uint32_t lo32 = 0, nm1 = 0, span = 0;
     auto warp_props = [&]() {
@@ -486,33 +551,12 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     const uint32_t tmin = (32u * a.elem_bytes + 127u) / 128u;       // R11
     const uint64_t Tl = DEPTH == 1 ? T0 : DEPTH == 2 ? T1 : DEPTH == 3 ? T2 : 1;
     const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
-    uint64_t m = off / Mk;
+    uint64_t m = udiv(off, Mk);
     uint64_t tt = off - m * Mk;
     if (MODE != 0 && closed_form && nest.par_dims == 1) {
-        // UNIFORM FLAGS, whole access (see below): a 1-D parallel stride g of 0 or
-        // >= 128 bytes gives every active lane after the first a line and a sector
-        // flag (g >= 128) or none (g = 0) in every warp-access, so a warp-rep with
-        // n active lanes has lines = sectors = 1 + (g ? n - 1 : 0) -- no lane work.
         const uint64_t g = uabs(a.c_par[0]);
-        if (g == 0 || g >= 128) {
-            WarpIter it;
-            warp_seek(it, m, P, B);
-            while (cnt > 0) {
-                const uint32_t k = uint32_t(umin64(Mk - tt, cnt));
-                const uint32_t nl = g ? it.n - 1u : 0u;
-                acc.W += k;
-                acc.K += k;
-                acc.lk += k * nl;
-                acc.sk += k * nl;
-                if (nl + 1u <= tmin) acc.C += k;
-                else acc.uk += k * nl;
-                cnt -= k;
-                tt = 0;
-                if (cnt > 0) warp_next(it, P, B);
-            }
-            return;
-        }
-        count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, cnt, lane, tmin, acc);
+        if (g == 0 || g >= 128) count_uniform(P, B, Mk, m, tt, cnt, g != 0, tmin, lane, acc);
+        else count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, cnt, lane, tmin, acc);
         return;
     }
     // inner indices, last fastest

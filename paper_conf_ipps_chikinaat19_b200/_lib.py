@@ -18,6 +18,7 @@ SEL_F_NO_DEDUP = 1
 SEL_F_MATCH_ANY = 2
 SEL_F_SCALAR = 4
 SEL_F_EXPAND_ALL = 8
+SEL_F_NO_RESIDUE_CLASSES = 16
 DECISION_CPU, DECISION_GPU, DECISION_INVALID = 0, 1, 0xFF
 
 
@@ -76,7 +77,7 @@ class Stats(ctypes.Structure):
     _fields_ = [("n_candidates", ctypes.c_uint64), ("n_problems", ctypes.c_uint64),
                 ("wa_analysed", ctypes.c_uint64), ("wa_covered", ctypes.c_uint64),
                 ("n_invalid", ctypes.c_uint64), ("wa_closed_form", ctypes.c_uint64),
-                ("wa_arith_lanes", ctypes.c_uint64), ("_reserved", ctypes.c_uint64 * 1)]
+                ("wa_arith_lanes", ctypes.c_uint64), ("wa_residue_classes", ctypes.c_uint64)]
 
 
 RECORDS = (DeviceParams, Access, Nest, Launch, Candidate, Counts)

@@ -38,6 +38,10 @@
 namespace sel {
 
 constexpr uint64_t kMaxChunk = 1ull << 20;   // WAs per chunk: keeps all accumulators 32-bit
+#ifndef SEL_HIST_MIN_MK
+#define SEL_HIST_MIN_MK 32
+#endif
+constexpr uint64_t kHistMinMk = SEL_HIST_MIN_MK;   // inner tuples per warp-rep below which count_arith is cheaper
 
 struct CountArgs {
     const sel_nest* nests;
@@ -50,6 +54,7 @@ struct CountArgs {
     WsHeader* hdr;
     uint32_t one;                       // 1 at run time: keeps adds as IMAD on the FMA pipe
     uint32_t closed_form;               // resolve warp-reps with uniform lane flags in closed form
+    uint32_t residue_classes;           // whole arithmetic-lane warp-reps by residue classes (count_hist)
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -63,8 +68,21 @@ struct Acc {
     uint32_t lf, sf, uf;             // per lane
     uint32_t cc;                     // per lane: coalesced WAs (arithmetic-lane path)
     uint32_t W, C, lk, sk, uk;       // uniform
-    uint32_t K, Q;                   // uniform statistics: WAs in closed form / arithmetic-lane path
+    uint32_t K, Q, H;                // uniform statistics: WAs in closed form / arithmetic lanes / residue classes
 };
+// Per-lane partial sums returned by the out-of-line 1-D paths (by value, so
+// the caller's accumulators stay in registers): line flags, sector flags,
+// coalesced WAs, line flags of uncoalesced WAs, WAs done lane by lane.
+struct Part {
+    uint32_t lf, sf, cc, uf, q;
+};
+__device__ __forceinline__ void add_part(Acc& acc, const Part& p) {
+    acc.lf += p.lf;
+    acc.sf += p.sf;
+    acc.cc += p.cc;
+    acc.uf += p.uf;
+}
+
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -341,7 +359,7 @@ __device__ __forceinline__ void warp_seek(WarpIter& it, uint64_t m, uint64_t P, 
         it.blk_end = ~0ull;
     } else {
         const uint32_t wpb = (B + 31) >> 5;
-        const uint64_t kb = m / wpb;
+        const uint64_t kb = udiv(m, wpb);
         const uint32_t w = uint32_t(m - kb * wpb);
         it.p0 = kb * B + 32ull * w;
         it.blk_end = (kb + 1) * B;
@@ -373,12 +391,6 @@ __device__ __forceinline__ int64_t lane_address(const sel_nest& nest, const sel_
     return a.base + a.c_par[0] * int64_t(p / nest.P1) + a.c_par[1] * int64_t(p % nest.P1);
 }
 
-// a / b with a 32-bit fast path (the common case: both operands below 2^32)
-__device__ __forceinline__ uint64_t udiv(uint64_t a, uint64_t b) {
-    if (a < b) return 0;
-    if (((a | b) >> 32) == 0) return uint32_t(a) / uint32_t(b);
-    return a / b;
-}
 
 // ------------------------------------------------------------- uniform flags
 // A 1-D parallel stride g of 0 or >= 128 bytes gives every active lane after
@@ -387,8 +399,8 @@ __device__ __forceinline__ uint64_t udiv(uint64_t a, uint64_t b) {
 // lanes has lines = sectors = 1 + (g ? n - 1 : 0) in all of its warp-accesses.
 // Lane l adds up warp-reps m0 + l, m0 + l + 32, ... of the chunk (closed form,
 // no expansion).
-__device__ void count_uniform(uint64_t P, uint32_t B, uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt,
-                              bool flags, uint32_t tmin, int lane, Acc& acc) {
+__device__ __noinline__ Part count_uniform(uint64_t P, uint32_t B, uint64_t Mk, uint64_t m0, uint64_t tt,
+                                           uint32_t cnt, bool flags, uint32_t tmin, int lane) {
     const uint64_t start = tt, end = tt + cnt;           // instances relative to warp-rep m0
     const uint64_t nw = udiv(end - 1, Mk) + 1;           // warp-reps touched
     const bool blocked = (B & 31u) != 0;
@@ -423,12 +435,7 @@ __device__ void count_uniform(uint64_t P, uint32_t B, uint64_t Mk, uint64_t m0, 
         if (nl + 1u <= tmin) cc += k;                     // R11
         else uf += k * nl;
     }
-    acc.lf += lf;
-    acc.sf += lf;
-    acc.cc += cc;
-    acc.uf += uf;
-    acc.W += cnt;
-    acc.K += cnt;
+    return Part{lf, lf, cc, uf, 0u};
 }
 
 // ------------------------------------------------------------- arithmetic lanes
@@ -444,9 +451,9 @@ __device__ void count_uniform(uint64_t P, uint32_t B, uint64_t Mk, uint64_t m0, 
 // l + 32, ... of the chunk, walking (warp-rep, inner tuple) as a mixed-radix
 // counter), 32 warp-accesses per warp instruction instead of one.
 template <int DEPTH>
-__device__ void count_arith(const sel_access& a, uint64_t P, uint32_t B, uint64_t T0, uint64_t T1, uint64_t T2,
-                            uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt, int lane, uint32_t tmin,
-                            Acc& acc) {
+__device__ __noinline__ Part count_arith(const sel_access& a, uint64_t P, uint32_t B, uint64_t T0, uint64_t T1,
+                                         uint64_t T2, uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt, int lane,
+                                         uint32_t tmin) {
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
@@ -532,12 +539,247 @@ __device__ void count_arith(const sel_access& a, uint64_t P, uint32_t B, uint64_
             warp_props();
         }
     }
-    acc.lf += lf;
-    acc.sf += sf;
-    acc.uf += uf;
-    acc.cc += cc;
-    acc.W += cnt;
-    acc.Q += cnt;
+    return Part{lf, sf, cc, uf, cnt};
+}
+
+// ------------------------------------------------------------- residue classes
+// Within one full warp-rep of an arithmetic-lane access (above) every
+// warp-access is fixed by r = (lo + D) mod 128, and D = sum_j k_j i_j.  So the
+// warp-rep's sums over its Mk inner tuples are  sum_rho h[rho] * f(lo + rho),
+// h[rho] = #{tuples : D = rho (mod 128)} -- the same integers as the tuple
+// by tuple sum, grouped by residue.  Addresses are multiples of the element
+// size E (V5), so h lives on the R = 128/E residues rho = s*E (slot s).
+//
+// h of one loop (k, T): k*i mod 128 has period pi = 128 / gcd(k mod 128, 128),
+// distinct over i < pi; residue k*i (i < min(T, pi)) occurs ceil((T - i)/pi)
+// times.  Nested loops convolve (cyclically, mod 128) the one-loop histograms.
+__device__ __forceinline__ uint32_t loop_period_log2(uint32_t k) {   // log2 pi
+    const uint32_t km = k & 127u;
+    return km == 0 ? 0u : 7u - uint32_t(__ffs(km) - 1);
+}
+
+// h <- histogram of one loop (k, T), T >= 1; smem, R slots of 2^sh bytes
+__device__ __forceinline__ void hist_one(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane) {
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++)
+        if (lane + 32u * j < R) h[lane + 32u * j] = 0;
+    __syncwarp();
+    const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
+    const uint32_t n = T < pi ? T : pi;                         // <= 128
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++) {
+        const uint32_t i = lane + 32u * j;
+        if (i < n) h[((k * i) & 127u) >> sh] = (T - i + pi - 1u) >> lp;
+    }
+    __syncwarp();
+}
+
+// h <- h (*) histogram of loop (k, T): out[rho] = sum_i cnt(i) h[rho - k i]
+__device__ __forceinline__ void hist_conv(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane) {
+    const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
+    const uint32_t n = T < pi ? T : pi;
+    uint32_t o[4] = {0u, 0u, 0u, 0u};
+    for (uint32_t i = 0; i < n; i++) {
+        const uint32_t c = (T - i + pi - 1u) >> lp;
+        const uint32_t off = k * i;
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const uint32_t s = uint32_t(lane) + 32u * j;
+            if (s < R) o[j] += c * h[(((s << sh) - off) & 127u) >> sh];
+        }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+        const uint32_t s = uint32_t(lane) + 32u * j;
+        if (s < R) h[s] = o[j];
+    }
+    __syncwarp();
+}
+
+// `mult` warp-reps whose lowest lane address is lo (mod 128) with nm1 + 1
+// active lanes: lane sums over the residues (same integers as count_arith)
+__device__ __forceinline__ void hist_eval(const uint32_t* h, uint32_t R, uint32_t sh, uint32_t lo, uint32_t nm1,
+                                          uint32_t g, uint32_t tmin, uint32_t mult, int lane, uint32_t& lf,
+                                          uint32_t& sf, uint32_t& cc, uint32_t& uf) {
+    const uint32_t span = nm1 * g;
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++) {
+        const uint32_t s = lane + 32u * j;
+        if (s >= R) break;
+        const uint32_t w = h[s] * mult;
+        const uint32_t r = (lo + (s << sh)) & 127u;
+        const uint32_t nl = (r + span) >> 7;                    // lines - 1
+        const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
+        lf += w * nl;
+        sf += w * ns;
+        if (nl < tmin) cc += w;                                 // R11
+        else uf += w * nl;
+    }
+}
+
+// WAs [tt, tt + cnt) from warp-rep m0 of a 1-D access with lane stride
+// 0 < g < 128: head and tail fragments of a warp-rep lane by lane
+// (count_arith), whole warp-reps by residue classes.
+template <int DEPTH>
+__device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_t B, uint64_t T0, uint64_t T1,
+                                        uint64_t T2, uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt, int lane,
+                                        uint32_t tmin, uint32_t* h) {
+    uint64_t m = m0;
+    Part out{0u, 0u, 0u, 0u, 0u};
+    auto add = [&](const Part& p) { out.lf += p.lf; out.sf += p.sf; out.cc += p.cc; out.uf += p.uf; out.q += p.q; };
+    if (tt > 0) {                                               // head: rest of warp-rep m0
+        const uint32_t k = uint32_t(umin64(Mk - tt, cnt));
+        add(count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, k, lane, tmin));
+        cnt -= k;
+        m++;
+        if (cnt == 0) return out;
+    }
+    const uint32_t Mk32 = uint32_t(Mk);                         // Mk <= cnt <= kMaxChunk here
+    const uint32_t nfull = cnt / Mk32;
+    const uint32_t rest = cnt - nfull * Mk32;
+    if (nfull) {
+        const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
+        const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
+                       k2 = uint32_t(uint64_t(a.c_inner[2]));
+        if (DEPTH == 1) hist_one(h, R, sh, k0, uint32_t(T0), lane);
+        if (DEPTH == 2) { hist_one(h, R, sh, k1, uint32_t(T1), lane); hist_conv(h, R, sh, k0, uint32_t(T0), lane); }
+        if (DEPTH == 3) {
+            hist_one(h, R, sh, k2, uint32_t(T2), lane);
+            hist_conv(h, R, sh, k1, uint32_t(T1), lane);
+            hist_conv(h, R, sh, k0, uint32_t(T0), lane);
+        }
+        const int64_t c0 = a.c_par[0];
+        const uint32_t g = uint32_t(uabs(c0));
+        const bool neg = c0 < 0;
+        const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
+        uint32_t lf = 0, sf = 0, cc = 0, uf = 0;
+        if ((B & 31u) == 0) {
+            // warp-rep j: p0 = 32 j, all 32 lanes active except the last one of P;
+            // lo mod 128 of a full warp-rep depends on j mod 4 only
+            const uint64_t nfl = P >> 5;                        // warp-reps with 32 active lanes
+            const uint64_t e = m + nfull;
+            const uint64_t ef = e < nfl ? e : (nfl > m ? nfl : m);
+            const uint64_t nf = ef - m;                         // full-lane warp-reps in [m, e)
+            for (uint32_t j = 0; j < 4; j++) {
+                // #{x in [m, m + nf) : x = j (mod 4)}
+                const uint64_t first = m + ((j - uint32_t(m)) & 3u);
+                const uint32_t cntj = first < m + nf ? uint32_t((m + nf - 1 - first) / 4 + 1) : 0u;
+                if (cntj == 0) continue;
+                const uint32_t lo = base32 + c032 * (32u * uint32_t(first)) + (neg ? c032 * 31u : 0u);
+                hist_eval(h, R, sh, lo, 31u, g, tmin, cntj, lane, lf, sf, cc, uf);
+            }
+            if (ef < e) {                                       // the partial last warp-rep of P
+                const uint32_t nm1 = uint32_t(P - 32ull * ef) - 1u;
+                const uint32_t lo = base32 + c032 * (32u * uint32_t(ef)) + (neg ? c032 * nm1 : 0u);
+                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf);
+            }
+        } else {
+            const uint32_t wpb = (B + 31u) >> 5;
+            uint64_t kb = udiv(m, wpb);
+            uint32_t w = uint32_t(m - kb * wpb);
+            for (uint32_t x = 0; x < nfull; x++) {
+                const uint64_t p0 = kb * B + 32ull * w;
+                const uint64_t pe = umin64(umin64(p0 + 32, (kb + 1) * uint64_t(B)), P);
+                const uint32_t nm1 = uint32_t(pe - p0) - 1u;
+                const uint32_t lo = base32 + c032 * uint32_t(p0) + (neg ? c032 * nm1 : 0u);
+                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf);
+                if (++w == wpb) { w = 0; kb++; }
+            }
+        }
+        add(Part{lf, sf, cc, uf, 0u});
+        __syncwarp();                                           // h is reused by the next access
+    }
+    if (rest) add(count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m + nfull, 0, rest, lane, tmin));
+    return out;
+}
+
+// ------------------------------------------------------------- whole accesses
+// When a chunk holds all WR * Mk warp-accesses of an access (the common case:
+// a chunk spans many small problems) the warp-reps need not be walked: by R8
+// and R9 they fall into at most three lane-count classes, computed once per
+// problem -- n32 warp-reps with 32 active lanes, nA with B mod 32 lanes (the
+// last warp of every complete block when 32 does not divide B) and at most
+// one with the last lanes of P.
+struct RepClasses {
+    uint64_t n32, nA;
+    uint32_t lanesA, lanesR;        // 0: class empty
+};
+__device__ __forceinline__ RepClasses rep_classes(uint64_t P, uint32_t B) {
+    RepClasses c;
+    if ((B & 31u) == 0) {
+        c.n32 = P >> 5;
+        c.nA = 0;
+        c.lanesA = 0;
+        c.lanesR = uint32_t(P & 31u);
+    } else {
+        const uint64_t nbf = udiv(P, B);                    // complete blocks
+        const uint32_t rem = uint32_t(P - nbf * B);         // iterations of the last, incomplete block
+        c.n32 = nbf * ((B - 1u) >> 5) + (rem >> 5);
+        c.nA = nbf;
+        c.lanesA = B & 31u;
+        c.lanesR = rem & 31u;
+    }
+    return c;
+}
+
+// Uniform lane flags over a whole access: a warp-rep with n active lanes has
+// lines = sectors = 1 + (flags ? n - 1 : 0) in each of its Mk warp-accesses
+// (count_uniform); warp-uniform accumulators.
+__device__ __forceinline__ void uniform_whole(const RepClasses& rc, uint32_t Mk, bool flags, uint32_t tmin,
+                                              Acc& acc) {
+    auto cls = [&](uint32_t lanes, uint32_t reps) {
+        const uint32_t w = reps * Mk;                       // <= WR * Mk <= kMaxChunk
+        const uint32_t nl = flags ? lanes - 1u : 0u;
+        acc.lk += w * nl;
+        acc.sk += w * nl;
+        if (nl + 1u <= tmin) acc.C += w;                    // R11
+        else acc.uk += w * nl;
+    };
+    if (rc.n32) cls(32u, uint32_t(rc.n32));
+    if (rc.nA) cls(rc.lanesA, uint32_t(rc.nA));
+    if (rc.lanesR) cls(rc.lanesR, 1u);
+}
+
+// Residue classes over a whole access (count_hist) when the lowest lane
+// address mod 128 of a warp-rep depends only on its lane count (32 | B with
+// 32 c = 0 mod 128, or B c = 32 c = 0 mod 128), or, for 32 | B, on the
+// warp-rep index mod 4: the histogram is built once and evaluated once per
+// class.  Runtime depth (0..3).
+__device__ __forceinline__ Part count_hist_whole(const sel_access& a, int depth, uint32_t T0, uint32_t T1,
+                                                 uint32_t T2, RepClasses rc, uint32_t tmin, uint32_t* h, int lane) {
+    const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
+    const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
+                   k2 = uint32_t(uint64_t(a.c_inner[2]));
+    if (depth == 0) hist_one(h, R, sh, 0u, 1u, lane);
+    else if (depth == 1) hist_one(h, R, sh, k0, T0, lane);
+    else if (depth == 2) { hist_one(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+    else { hist_one(h, R, sh, k2, T2, lane); hist_conv(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+    const int64_t c0 = a.c_par[0];
+    const uint32_t g = uint32_t(uabs(c0));
+    const bool neg = c0 < 0;
+    const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
+    Part o{0u, 0u, 0u, 0u, 0u};
+    // lowest lane address of a warp-rep starting at iteration p0 with n lanes
+    auto lo_of = [&](uint32_t p0, uint32_t n) { return base32 + c032 * p0 + (neg ? c032 * (n - 1u) : 0u); };
+    if (rc.n32) {
+        if (((32u * c032) & 127u) == 0) {
+            hist_eval(h, R, sh, lo_of(0u, 32u), 31u, g, tmin, uint32_t(rc.n32), lane, o.lf, o.sf, o.cc, o.uf);
+        } else {                                            // 32 | B here: warp-rep j starts at 32 j
+            for (uint32_t j = 0; j < 4; j++) {
+                const uint32_t cj = uint32_t((rc.n32 + 3u - j) >> 2);   // #{x < n32 : x = j mod 4}
+                if (cj) hist_eval(h, R, sh, lo_of(32u * j, 32u), 31u, g, tmin, cj, lane, o.lf, o.sf, o.cc, o.uf);
+            }
+        }
+    }
+    if (rc.nA) hist_eval(h, R, sh, lo_of(0u, rc.lanesA), rc.lanesA - 1u, g, tmin, uint32_t(rc.nA), lane, o.lf, o.sf,
+                         o.cc, o.uf);
+    if (rc.lanesR) {                                        // the last warp-rep of P starts at 32 n32 (32 | B)
+        const uint32_t p0 = rc.nA ? 0u : uint32_t(32u * rc.n32);
+        hist_eval(h, R, sh, lo_of(p0, rc.lanesR), rc.lanesR - 1u, g, tmin, 1u, lane, o.lf, o.sf, o.cc, o.uf);
+    }
+    __syncwarp();                                           // h is reused by the next access
+    return o;
 }
 
 // ------------------------------------------------------------- per access
@@ -553,17 +795,11 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     const int64_t cl = DEPTH == 1 ? a.c_inner[0] : DEPTH == 2 ? a.c_inner[1] : DEPTH == 3 ? a.c_inner[2] : 0;
     uint64_t m = udiv(off, Mk);
     uint64_t tt = off - m * Mk;
-    if (MODE != 0 && closed_form && nest.par_dims == 1) {
-        const uint64_t g = uabs(a.c_par[0]);
-        if (g == 0 || g >= 128) count_uniform(P, B, Mk, m, tt, cnt, g != 0, tmin, lane, acc);
-        else count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, cnt, lane, tmin, acc);
-        return;
-    }
     // inner indices, last fastest
     uint64_t i0 = 0, i1 = 0, i2 = 0;
     if (DEPTH == 1) { i0 = tt; }
-    if (DEPTH == 2) { i1 = tt % T1; i0 = tt / T1; }
-    if (DEPTH == 3) { i2 = tt % T2; const uint64_t r = tt / T2; i1 = r % T1; i0 = r / T1; }
+    if (DEPTH == 2) { i0 = udiv(tt, T1); i1 = tt - i0 * T1; }
+    if (DEPTH == 3) { const uint64_t r = udiv(tt, T2); i2 = tt - r * T2; i0 = udiv(r, T1); i1 = r - i0 * T1; }
     WarpIter it;
     warp_seek(it, m, P, B);
     while (cnt > 0) {
@@ -670,47 +906,126 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
     }
     if (acc.K && lane == 5) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)acc.K);
     if (acc.Q && lane == 6) atomicAdd((unsigned long long*)&a.hdr->stats.wa_arith_lanes, (unsigned long long)acc.Q);
+    if (acc.H && lane == 7) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)acc.H);
     acc = Acc{};
 }
 
+// Cold and warm paths, out of line so the hot per-problem loop stays compact
+// in the instruction cache.  General 1-D access slice (chunk boundaries,
+// blocks that break the residue classes): uniform flags, residue classes
+// with head/tail fragments, or arithmetic lanes.
+struct Part1 {
+    Part p;
+    uint32_t uniform;                                       // 1: the WAs were uniform-flag closed form
+};
+__device__ __noinline__ Part1 count_1d_general(const sel_access* ap, uint64_t P, uint32_t B, uint64_t T0,
+                                               uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t t,
+                                               uint32_t tc, int lane, uint32_t* hist) {
+    const sel_access ac = *ap;
+    const int d = ac.depth;
+    const uint64_t g = uabs(ac.c_par[0]);
+    const uint64_t m = off ? udiv(off, Mk) : 0, tt = off - m * Mk;
+    if (g == 0 || g >= 128) return Part1{count_uniform(P, B, Mk, m, tt, t, g != 0, tc, lane), 1u};
+    const bool hs = d >= 1 && hist && Mk >= kHistMinMk;
+    Part p;
+    switch (d) {
+    case 0: p = count_arith<0>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc); break;
+    case 1: p = hs ? count_hist<1>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc, hist)
+                   : count_arith<1>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc); break;
+    case 2: p = hs ? count_hist<2>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc, hist)
+                   : count_arith<2>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc); break;
+    default: p = hs ? count_hist<3>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc, hist)
+                    : count_arith<3>(ac, P, B, T0, T1, T2, Mk, m, tt, t, lane, tc); break;
+    }
+    return Part1{p, 0u};
+}
+
+// Lane-by-lane expansion (collapse(2) accesses, SEL_F_EXPAND_ALL, MATCH).
 template <int MODE>
-__device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane) {
-    const sel_nest nest = a.nests[a.prob_nest[q]];
+__device__ __noinline__ Acc expand_access(const sel_nest* np, const sel_access* ap, uint64_t P, uint32_t B,
+                                          uint64_t T0, uint64_t T1, uint64_t T2, uint64_t Mk, uint64_t off, uint32_t t,
+                                          int lane, uint32_t one, uint32_t closed_form, Acc acc) {
+    const sel_nest nest = *np;
+    const sel_access ac = *ap;
+    const int d = ac.depth;
+    const int tc = (32 * int(ac.elem_bytes) + 127) / 128;       // tmin (R11): 1, 2 or 4
+#define SEL_DISPATCH(M, TCV)                                                                                  \
+    switch (d) {                                                                                              \
+    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, one, closed_form, acc); break;  \
+    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, one, closed_form, acc); break;  \
+    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, one, closed_form, acc); break;  \
+    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, one, closed_form, acc); break; \
+    }
+    if (MODE == 0) {
+        SEL_DISPATCH(0, 1)
+    } else if (tc == 1) {
+        SEL_DISPATCH(MODE, 1)
+    } else if (tc == 2) {
+        SEL_DISPATCH(MODE, 2)
+    } else {
+        SEL_DISPATCH(MODE, 4)
+    }
+#undef SEL_DISPATCH
+    return acc;
+}
+
+// WAs [off, off + take) of problem q, access by access.
+template <int MODE>
+__device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane, uint32_t* hist) {
+    const sel_nest* np = a.nests + a.prob_nest[q];
+    const sel_nest nest = *np;
     const uint32_t B = a.prob_B[q];
     const uint64_t WR = a.prob_WR[q];
     const uint64_t P = nest.P0 * nest.P1;
     const uint64_t T0 = eff_trip(nest.trip[0]), T1 = eff_trip(nest.trip[1]), T2 = eff_trip(nest.trip[2]);
+    const uint64_t Mks[4] = {1, T0, T0 * T1, T0 * T1 * T2};
+    const bool one_d = MODE != 0 && a.closed_form && nest.par_dims == 1;
+    RepClasses rc{0, 0, 0u, 0u};
+    if (one_d) rc = rep_classes(P, B);
     Acc acc{};
-    for (uint32_t k = 0; k < nest.n_access && take > 0; k++) {
-        const sel_access ac = a.acc[nest.access_off + k];
+    const sel_access* ap = a.acc + nest.access_off;
+    for (uint32_t k = 0; k < nest.n_access && take > 0; k++, ap++) {
+        const sel_access ac = *ap;
         const int d = ac.depth;
-        const uint64_t Mk = d == 0 ? 1 : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
+        const uint64_t Mk = d == 0 ? Mks[0] : d == 1 ? Mks[1] : d == 2 ? Mks[2] : Mks[3];
         const uint64_t Wk = WR * Mk;
         if (off >= Wk) {
             off -= Wk;
             continue;
         }
         const uint32_t t = uint32_t(umin64(Wk - off, take));
-        const int tc = (32 * int(ac.elem_bytes) + 127) / 128;     // tmin (R11): 1, 2 or 4
-#define SEL_DISPATCH(M, TCV)                                                                          \
-    switch (d) {                                                                                      \
-    case 0: count_access<M, 0, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
-    case 1: count_access<M, 1, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
-    case 2: count_access<M, 2, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;        \
-    default: count_access<M, 3, TCV>(nest, ac, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc); break;       \
-    }
-        if (MODE == 0) {
-            SEL_DISPATCH(0, 1)
-        } else if (tc == 1) {
-            SEL_DISPATCH(MODE, 1)
-        } else if (tc == 2) {
-            SEL_DISPATCH(MODE, 2)
-        } else {
-            SEL_DISPATCH(MODE, 4)
-        }
-#undef SEL_DISPATCH
+        acc.W += t;
         take -= t;
+        if (!one_d) {
+            acc.W -= t;                                         // expand_access accumulates W itself
+            acc = expand_access<MODE>(np, ap, P, B, T0, T1, T2, Mk, off, t, lane, a.one, a.closed_form, acc);
+            off = 0;
+            continue;
+        }
+        // 1-D parallel access: lane addresses an arithmetic progression
+        const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // tmin (R11)
+        const uint32_t g = uint32_t(umin64(uabs(ac.c_par[0]), 128));
+        const bool whole = off == 0 && t == Wk;
+        const uint64_t off0 = off;
         off = 0;
+        if (whole && (g == 0 || g == 128)) {
+            uniform_whole(rc, uint32_t(Mk), g != 0, tc, acc);
+            acc.K += t;
+            continue;
+        }
+        const uint32_t cB = uint32_t(uint64_t(ac.c_par[0])) * B;
+        if (whole && hist && ((B & 31u) == 0 || (((cB | (32u * g)) & 127u) == 0))) {
+            add_part(acc, count_hist_whole(ac, d, uint32_t(T0), uint32_t(T1), uint32_t(T2), rc, tc, hist, lane));
+            acc.H += t;
+            continue;
+        }
+        const Part1 r = count_1d_general(ap, P, B, T0, T1, T2, Mk, off0, t, tc, lane, hist);
+        add_part(acc, r.p);
+        if (r.uniform) acc.K += t;
+        else {
+            acc.Q += r.p.q;
+            acc.H += t - r.p.q;
+        }
     }
     flush(a, q, acc, lane);
 }
@@ -724,6 +1039,8 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
 template <int MODE>
 __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
     const int lane = threadIdx.x & 31;
+    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][128];
+    uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;
     const uint64_t base = a.hdr->w_begin, end = a.hdr->w_end;   // this call's slice of [0, prefix[nq])
@@ -749,7 +1066,7 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
                 continue;
             }
             const uint32_t take = uint32_t(umin64(Wq - off, len));
-            count_problem<MODE>(a, q, off, take, lane);
+            count_problem<MODE>(a, q, off, take, lane, hist);
             len -= take;
             off = 0;
             q++;
@@ -775,7 +1092,7 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
     (void)max_problems;
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
-                (flags & SEL_F_EXPAND_ALL) ? 0u : 1u};
+                (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u};
     prof_before_count(s);
     if (mode == 0) k_count<0><<<count_grid<0>(), SEL_COUNT_THREADS, 0, s>>>(a);
     else if (mode == 1) k_count<1><<<count_grid<1>(), SEL_COUNT_THREADS, 0, s>>>(a);

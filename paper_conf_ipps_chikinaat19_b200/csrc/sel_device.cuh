@@ -69,7 +69,16 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
 __device__ __forceinline__ uint64_t eff_trip(uint32_t t) {
     return t == SEL_TRIP_UNKNOWN ? 128ull : uint64_t(t);
 }
-__device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return a / b + (a % b != 0); }
+// a / b with a 32-bit fast path (the common case: both operands below 2^32;
+// the 64-bit division is a long software sequence)
+__device__ __forceinline__ uint64_t udiv(uint64_t a, uint64_t b) {
+    if (((a | b) >> 32) == 0) return uint32_t(a) / uint32_t(b);
+    return a / b;
+}
+__device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) {
+    const uint64_t q = udiv(a, b);
+    return q + (a - q * b != 0);
+}
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ uint64_t smul(uint64_t a, uint64_t b) {
     if (a == 0 || b == 0) return 0;

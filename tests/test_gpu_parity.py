@@ -304,7 +304,7 @@ def _random_medium_batch(seed, n):
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 2, 4, 8, 12])
+@pytest.mark.parametrize("flags", [0, 2, 4, 8, 12, 16])
 def test_random_medium_nests(sel, flags):
     b = _random_medium_batch(123 + flags, 1500)
     ref = oracle.evaluate(b)
@@ -362,7 +362,7 @@ def _uniform_gap_batch():
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 4, 8, 1])
+@pytest.mark.parametrize("flags", [0, 4, 8, 1, 16])
 def test_uniform_flag_closed_form(sel, flags):
     b = _uniform_gap_batch()
     ref = oracle.evaluate(b)
@@ -371,10 +371,11 @@ def test_uniform_flag_closed_form(sel, flags):
     assert_parity(g, ref, ctx=f"uniform-gap flags={flags}")
     st = g["stats"]
     if flags & 8:
-        assert st["wa_closed_form"] == 0 and st["wa_arith_lanes"] == 0
+        assert st["wa_closed_form"] == 0 and st["wa_arith_lanes"] == 0 and st["wa_residue_classes"] == 0
     else:
         assert 0 < st["wa_closed_form"] and 0 < st["wa_arith_lanes"]
-        assert st["wa_closed_form"] + st["wa_arith_lanes"] < st["wa_analysed"]     # collapse(2) expands
+        assert (st["wa_closed_form"] + st["wa_arith_lanes"] + st["wa_residue_classes"]
+                < st["wa_analysed"])                                              # collapse(2) expands
 
 
 def test_closed_form_share_c5_slice(sel):
@@ -385,3 +386,61 @@ def test_closed_form_share_c5_slice(sel):
     assert (g0["counts"] == g8["counts"]).all() and (g0["cycles"] == g8["cycles"]).all()
     assert g0["stats"]["wa_analysed"] == g8["stats"]["wa_analysed"]
     assert g0["stats"]["wa_closed_form"] > g0["stats"]["wa_analysed"] // 2
+
+
+def _residue_class_batch(seed, n):
+    """1-D accesses with lane strides 0 < g < 128 and long inner loops, so
+    whole warp-reps are summed by residue class: every element
+    size, odd / even / negative / multiple-of-128 inner coefficients (loop
+    periods 1..128), depth 1-3, inner trips around the 32-tuple threshold,
+    P with a partial last warp, blocks that 32 does and does not divide, a
+    grid cap (#OMP_Rep > 1) and chunk boundaries inside warp-reps."""
+    rnd = random.Random(seed)
+    Bs = [32, 64, 256, 48, 200, 100, 1000, 33]
+    launches = np.zeros(len(Bs), gen.LAUNCH_DTYPE)
+    for i, B in enumerate(Bs):
+        launches[i] = (B, rnd.choice([1, 5, 65535]), 0, 0)
+    items = []
+    for _ in range(n):
+        depth = rnd.choice([1, 2, 2, 3])
+        trip = [rnd.choice([1, 2, 7, 31, 32, 33, 64, 129, 300][: 9 - 3 * (depth - 1)]) for _ in range(depth)]
+        acc = []
+        for _ in range(rnd.randint(1, 4)):
+            e = rnd.choice([1, 2, 4, 8, 16])
+            g = e * rnd.randint(1, max(1, 127 // e))
+            cp = rnd.choice([g, -g, e, 2 * e])
+            d = rnd.randint(1, depth)
+
+            def coef():
+                return e * rnd.choice([0, 1, -1, 3, 5, 7, 8, 12, 16, 31, 32, 128, -96, 1000, 1030 + rnd.randint(0, 64)])
+            acc.append(gen.make_access(base=(1 << 34) + e * rnd.randint(-2000, 2000), c_par=[cp],
+                                       c_inner=[coef() for _ in range(d)], elem_bytes=e, depth=d))
+        items.append(dict(P0=rnd.choice([1, 31, 32, 33, 95, 96, 97, 500, 1000, 2049]), trip=trip, depth=depth,
+                          comp=[1.0] * (depth + 1), accesses=acc, launch=rnd.randrange(len(Bs)),
+                          device=rnd.randrange(4)))
+    return gen.custom_batch(items, launches_=launches)
+
+
+@pytest.mark.parametrize("flags", [0, 16, 4, 1, 8])
+def test_residue_classes(sel, flags):
+    b = _residue_class_batch(77 + flags, 1500)
+    ref = oracle.evaluate(b)
+    assert (ref["status"] == 0).all()
+    g = run_gpu(sel, b, flags)
+    assert_parity(g, ref, ctx=f"residue classes flags={flags}")
+    st = g["stats"]
+    if flags & (8 | 16):
+        assert st["wa_residue_classes"] == 0
+    else:
+        assert st["wa_residue_classes"] > 0 and st["wa_arith_lanes"] > 0   # arith: fragments, short rows
+
+
+def test_residue_classes_c5_slice(sel):
+    """c5 slice: residue-class counting agrees with lane-by-lane expansion
+    and with the arithmetic-lane path, counts and cycles bit for bit."""
+    b = gen.generate(5, 3000000, 3300000)
+    g0, g16, g8 = run_gpu(sel, b, 0), run_gpu(sel, b, 16), run_gpu(sel, b, 8)
+    for g in (g16, g8):
+        assert (g0["counts"] == g["counts"]).all() and (g0["cycles"] == g["cycles"]).all()
+        assert (g0["decision"] == g["decision"]).all()
+    assert g0["stats"]["wa_residue_classes"] > 0 and g16["stats"]["wa_residue_classes"] == 0

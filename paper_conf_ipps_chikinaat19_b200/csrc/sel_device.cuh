@@ -82,7 +82,7 @@ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) {
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ uint64_t smul(uint64_t a, uint64_t b) {
     if (a == 0 || b == 0) return 0;
-    return (a > ~0ull / b) ? ~0ull : a * b;
+    return __umul64hi(a, b) ? ~0ull : a * b;               // saturate on overflow
 }
 __device__ __forceinline__ uint64_t sadd(uint64_t a, uint64_t b) { return (a > ~0ull - b) ? ~0ull : a + b; }
 __device__ __forceinline__ uint64_t uabs(int64_t v) { return v < 0 ? 0ull - uint64_t(v) : uint64_t(v); }

@@ -154,9 +154,12 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
         const unsigned peers = __match_any_sync(inmask, key);
         const int leader = __ffs(peers) - 1;
         if (st == 0 && (threadIdx.x & 31) == leader) {
+            // open addressing from a hashed start slot (k_rank_slots sorts the slots
+            // afterwards, so positions do not matter): usually one CAS, not a chain
             uint32_t* s = slots + uint64_t(cd.nest_id) * kSlots;
+            const uint32_t h0 = (bc * 0x9E3779B1u) >> 29;
             for (int j = 0; j < kSlots; j++) {
-                uint32_t old = atomicCAS(s + j, 0u, bc);
+                const uint32_t old = atomicCAS(s + ((h0 + j) & (kSlots - 1)), 0u, bc);
                 if (old == 0u || old == bc) break;
             }
         }
@@ -201,8 +204,12 @@ __global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict_
     }
     if (pid == ~0ull) pid = nest_base[n_nests] + atomicAdd(&hdr->n_overflow, 1u);   // slot table full
     cand_pid[c] = uint32_t(pid);
-    prob_nest[pid] = cd.nest_id;      // identical values from every sharer
-    prob_B[pid] = bc;
+    // identical values from every sharer: one write per distinct problem of the warp
+    const unsigned peers = __match_any_sync(__activemask(), pid);
+    if ((threadIdx.x & 31) == __ffs(peers) - 1) {
+        prob_nest[pid] = cd.nest_id;
+        prob_B[pid] = bc;
+    }
 }
 
 __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_base, uint64_t n_nests,

@@ -19,6 +19,7 @@ SEL_F_MATCH_ANY = 2
 SEL_F_SCALAR = 4
 SEL_F_EXPAND_ALL = 8
 SEL_F_NO_RESIDUE_CLASSES = 16
+SEL_F_WARP_PROBLEMS = 32
 DECISION_CPU, DECISION_GPU, DECISION_INVALID = 0, 1, 0xFF
 
 

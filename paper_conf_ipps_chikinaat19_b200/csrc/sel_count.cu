@@ -38,6 +38,12 @@
 namespace sel {
 
 constexpr uint64_t kMaxChunk = 1ull << 20;   // WAs per chunk: keeps all accumulators 32-bit
+#ifndef SEL_COUNT_MIN_BLOCKS
+#define SEL_COUNT_MIN_BLOCKS 3
+#endif
+#ifndef SEL_COUNT_THREADS
+#define SEL_COUNT_THREADS 256
+#endif
 #ifndef SEL_HIST_MIN_MK
 #define SEL_HIST_MIN_MK 32
 #endif
@@ -55,6 +61,7 @@ struct CountArgs {
     uint32_t one;                       // 1 at run time: keeps adds as IMAD on the FMA pipe
     uint32_t closed_form;               // resolve warp-reps with uniform lane flags in closed form
     uint32_t residue_classes;           // whole arithmetic-lane warp-reps by residue classes (count_hist)
+    unsigned long long* queue;          // small problems handed from k_lane_problems to k_queue
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -741,6 +748,64 @@ __device__ __forceinline__ void uniform_whole(const RepClasses& rc, uint32_t Mk,
     if (rc.lanesR) cls(rc.lanesR, 1u);
 }
 
+// h <- residue histogram of the access's inner offsets (runtime depth 0..3)
+__device__ __forceinline__ void hist_build(uint32_t* h, const sel_access& a, int depth, uint32_t T0, uint32_t T1,
+                                           uint32_t T2, uint32_t R, uint32_t sh, int lane) {
+    const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
+                   k2 = uint32_t(uint64_t(a.c_inner[2]));
+    if (depth == 0) hist_one(h, R, sh, 0u, 1u, lane);
+    else if (depth == 1) hist_one(h, R, sh, k0, T0, lane);
+    else if (depth == 2) { hist_one(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+    else { hist_one(h, R, sh, k2, T2, lane); hist_conv(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+}
+
+// Residue classes over a whole access when the warp-reps' lowest lane
+// addresses fall into many classes (32 does not divide B and B c != 0 mod
+// 128): one warp-rep PER LANE (p0, active lanes and lo from the block
+// geometry, R8/R9), each lane summing its warp-rep over the R residues of h.
+// Same integers as hist_eval per warp-rep.  WR <= kSmallMaxWR.
+__device__ __noinline__ Part count_hist_reps(const sel_access* ap, int depth, uint32_t T0, uint32_t T1, uint32_t T2,
+                                             uint32_t P, uint32_t B, uint32_t WR, uint32_t tmin, uint32_t* h,
+                                             int lane) {
+    const sel_access a = *ap;
+    const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
+    hist_build(h, a, depth, T0, T1, T2, R, sh, lane);
+    const int64_t c0 = a.c_par[0];
+    const uint32_t g = uint32_t(uabs(c0));
+    const bool neg = c0 < 0;
+    const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
+    const uint32_t wpb = (B + 31u) >> 5;
+    Part o{0u, 0u, 0u, 0u, 0u};
+    for (uint32_t m0 = 0; m0 < WR; m0 += 32) {
+        const uint32_t m = m0 + uint32_t(lane);
+        const bool act = m < WR;
+        uint32_t lo = 0, nm1 = 0;
+        if (act) {
+            const uint32_t kb = m / wpb, w = m - kb * wpb;
+            const uint32_t p0 = kb * B + 32u * w;
+            uint32_t pe = p0 + 32u;
+            pe = pe < (kb + 1u) * B ? pe : (kb + 1u) * B;
+            pe = pe < P ? pe : P;
+            nm1 = pe - p0 - 1u;
+            lo = base32 + c032 * p0 + (neg ? c032 * nm1 : 0u);
+        }
+        const uint32_t span = nm1 * g;
+        for (uint32_t s = 0; s < R; s++) {
+            const uint32_t w = h[s];                        // same slot on every lane: broadcast
+            if (w == 0 || !act) continue;
+            const uint32_t r = (lo + (s << sh)) & 127u;
+            const uint32_t nl = (r + span) >> 7;
+            const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
+            o.lf += w * nl;
+            o.sf += w * ns;
+            if (nl < tmin) o.cc += w;                       // R11
+            else o.uf += w * nl;
+        }
+    }
+    __syncwarp();                                           // h is reused by the next access
+    return o;
+}
+
 // Residue classes over a whole access (count_hist) when the lowest lane
 // address mod 128 of a warp-rep depends only on its lane count (32 | B with
 // 32 c = 0 mod 128, or B c = 32 c = 0 mod 128), or, for 32 | B, on the
@@ -749,12 +814,7 @@ __device__ __forceinline__ void uniform_whole(const RepClasses& rc, uint32_t Mk,
 __device__ __forceinline__ Part count_hist_whole(const sel_access& a, int depth, uint32_t T0, uint32_t T1,
                                                  uint32_t T2, RepClasses rc, uint32_t tmin, uint32_t* h, int lane) {
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
-    const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
-                   k2 = uint32_t(uint64_t(a.c_inner[2]));
-    if (depth == 0) hist_one(h, R, sh, 0u, 1u, lane);
-    else if (depth == 1) hist_one(h, R, sh, k0, T0, lane);
-    else if (depth == 2) { hist_one(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
-    else { hist_one(h, R, sh, k2, T2, lane); hist_conv(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+    hist_build(h, a, depth, T0, T1, T2, R, sh, lane);
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
@@ -971,7 +1031,7 @@ __device__ __noinline__ Acc expand_access(const sel_nest* np, const sel_access* 
 
 // WAs [off, off + take) of problem q, access by access.
 template <int MODE>
-__device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane, uint32_t* hist) {
+__device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane, uint32_t* hist) {
     const sel_nest* np = a.nests + a.prob_nest[q];
     const sel_nest nest = *np;
     const uint32_t B = a.prob_B[q];
@@ -1030,14 +1090,219 @@ __device__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint
     flush(a, q, acc, lane);
 }
 
-#ifndef SEL_COUNT_MIN_BLOCKS
-#define SEL_COUNT_MIN_BLOCKS 3
-#endif
-#ifndef SEL_COUNT_THREADS
-#define SEL_COUNT_THREADS 256
-#endif
+// ------------------------------------------------------------- lane-parallel problems
+// Whole 1-D problems inside a chunk, ONE PER LANE: the closed forms above are
+// scalar work per (problem, access) -- a warp doing them in lockstep issues
+// 32 copies of the same scalar instructions.  Lane l takes problem qa + l and
+// handles its uniform-flag accesses (lane-count classes) and its depth <= 1
+// residue-class accesses (<= 128 residues of one loop, evaluated per class in
+// the lane); at the first access that needs the warp (deeper loop nests, block
+// sizes whose warp-reps fall into many residue classes, collapse(2)) it hands
+// the rest of its problem to the warp (queue of <= 32 entries).
+struct LaneSums {
+    uint32_t W, L, S, C, U;
+};
+
+// uniform flags over a whole access, one lane (uniform_whole)
+__device__ __forceinline__ void lane_uniform(const RepClasses& rc, uint32_t Mk, bool flags, uint32_t tmin,
+                                             LaneSums& z) {
+    auto cls = [&](uint32_t lanes, uint32_t reps) {
+        const uint32_t w = reps * Mk;
+        const uint32_t nl = flags ? lanes : 1u;             // lines = sectors per WA
+        z.L += w * nl;
+        z.S += w * nl;
+        if (nl <= tmin) z.C += w;                           // R11
+        else z.U += w * nl;
+    };
+    if (rc.n32) cls(32u, uint32_t(rc.n32));
+    if (rc.nA) cls(rc.lanesA, uint32_t(rc.nA));
+    if (rc.lanesR) cls(rc.lanesR, 1u);
+}
+
+// residue classes of a depth <= 1 access over a whole problem, one lane:
+// sum_{i < min(T, pi)} cnt(i) f(lo + k i) per warp-rep class (count_hist_whole)
+__device__ __forceinline__ void lane_hist1(const sel_access& a, uint32_t T, const RepClasses& rc, uint32_t tmin,
+                                           LaneSums& z) {
+    const uint32_t k = a.depth ? uint32_t(uint64_t(a.c_inner[0])) : 0u;
+    const uint32_t TT = a.depth ? T : 1u;
+    const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
+    const uint32_t n = TT < pi ? TT : pi;
+    const int64_t c0 = a.c_par[0];
+    const uint32_t g = uint32_t(uabs(c0));
+    const bool neg = c0 < 0;
+    const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
+    auto cls = [&](uint32_t lo, uint32_t nm1, uint32_t mult) {
+        const uint32_t span = nm1 * g;
+        for (uint32_t i = 0; i < n; i++) {
+            const uint32_t w = ((TT - i + pi - 1u) >> lp) * mult;
+            const uint32_t r = (lo + k * i) & 127u;
+            const uint32_t nl = (r + span) >> 7;            // lines - 1
+            const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
+            z.L += w * (nl + 1u);
+            z.S += w * (ns + 1u);
+            if (nl < tmin) z.C += w;                        // R11
+            else z.U += w * (nl + 1u);
+        }
+    };
+    auto lo_of = [&](uint32_t p0, uint32_t nl) { return base32 + c032 * p0 + (neg ? c032 * (nl - 1u) : 0u); };
+    if (rc.n32) {
+        if (((32u * c032) & 127u) == 0) cls(lo_of(0u, 32u), 31u, uint32_t(rc.n32));
+        else
+            for (uint32_t j = 0; j < 4; j++) {
+                const uint32_t cj = uint32_t((rc.n32 + 3u - j) >> 2);
+                if (cj) cls(lo_of(32u * j, 32u), 31u, cj);
+            }
+    }
+    if (rc.nA) cls(lo_of(0u, rc.lanesA), rc.lanesA - 1u, uint32_t(rc.nA));
+    if (rc.lanesR) cls(lo_of(rc.nA ? 0u : uint32_t(32u * rc.n32), rc.lanesR), rc.lanesR - 1u, 1u);
+}
+
+// Small problems (k_problem_w: 1-D, W <= kSmallMaxW, WR <= kSmallMaxWR), one
+// per thread, grid-stride over this call's problem range.  A thread hands the
+// rest of its problem to the warp kernel (k_queue) at the first access that
+// needs a warp: entry = problem << 32 | WA offset of that access.
 template <int MODE>
-__global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(CountArgs a) {
+__global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ CountArgs a) {
+    const uint64_t q_end = a.hdr->small_end;
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    uint32_t sK = 0, sH = 0;                                // statistics: WAs by path
+    unsigned long long sW = 0;
+    for (uint64_t qb = a.hdr->small_begin + uint64_t(blockIdx.x) * blockDim.x; qb < q_end; qb += stride) {
+        const uint64_t q = qb + threadIdx.x;
+        uint32_t hmask = 0;                                 // accesses handed to the warp kernel
+        if (q < q_end && a.prefix[q + 1] == a.prefix[q]) {
+            const uint64_t WR64 = a.prob_WR[q];
+            const uint64_t Wq = WR64 * a.prob_cnt[q * kCntStride + 5];
+            if (Wq) {                                       // small (valid, outside the prefix)
+                sW += Wq;
+                const sel_nest nest = a.nests[a.prob_nest[q]];
+                const uint32_t B = a.prob_B[q];
+                const uint32_t WR = uint32_t(WR64);
+                const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
+                               T2 = uint32_t(eff_trip(nest.trip[2]));
+                const RepClasses rc = rep_classes(nest.P0, B);
+                LaneSums z{0u, 0u, 0u, 0u, 0u};
+                const sel_access* ap = a.acc + nest.access_off;
+                for (uint32_t k = 0; k < nest.n_access; k++, ap++) {
+                    if (k == 31) {                          // accesses 31, 32, ...: all to the warp kernel
+                        hmask |= 1u << 31;
+                        break;
+                    }
+                    const sel_access ac = *ap;
+                    const uint32_t d = ac.depth;
+                    const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
+                    const uint32_t Wk = WR * Mk;
+                    if (Wk == 0) continue;
+                    const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
+                    const uint32_t g = uint32_t(umin64(uabs(ac.c_par[0]), 128));
+                    if (g == 0 || g == 128) {
+                        lane_uniform(rc, Mk, g != 0, tc, z);
+                        sK += Wk;
+                    } else if (d <= 1 && a.residue_classes &&
+                               ((B & 31u) == 0 ||
+                                (((uint32_t(uint64_t(ac.c_par[0])) * B) | (32u * g)) & 127u) == 0)) {
+                        lane_hist1(ac, T0, rc, tc, z);
+                        sH += Wk;
+                    } else {
+                        hmask |= 1u << k;                   // the warp kernel counts access k
+                        continue;
+                    }
+                    z.W += Wk;
+                }
+                if (z.W) {
+                    unsigned long long* pc = a.prob_cnt + q * kCntStride;
+                    atomicAdd(pc + 0, (unsigned long long)z.W);
+                    atomicAdd(pc + 1, (unsigned long long)z.L);
+                    atomicAdd(pc + 2, (unsigned long long)z.S);
+                    atomicAdd(pc + 3, (unsigned long long)z.C);
+                    atomicAdd(pc + 4, (unsigned long long)z.U);
+                }
+            }
+        }
+        // warp-aggregated append to the queue
+        const bool enq = hmask != 0;
+        const unsigned m = __ballot_sync(kFull, enq);
+        if (m) {
+            unsigned long long base = 0;
+            const int lane = threadIdx.x & 31;
+            if (lane == __ffs(m) - 1) base = atomicAdd(&a.hdr->queue_len, (unsigned long long)__popc(m));
+            base = __shfl_sync(kFull, base, __ffs(m) - 1);
+            if (enq) a.queue[base + __popc(m & lanemask_lt())] = (q << 32) | hmask;
+        }
+    }
+    const uint32_t K = __reduce_add_sync(kFull, sK), H = __reduce_add_sync(kFull, sH);
+    unsigned long long Wt = sW;
+    for (int o = 16; o; o >>= 1) Wt += __shfl_xor_sync(kFull, Wt, o);
+    const int lane = threadIdx.x & 31;
+    if (K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)K);
+    if (H && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)H);
+    if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_analysed, Wt);
+}
+
+// The handed-over rest of small problems, one warp per queue entry.
+template <int MODE>
+__global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_queue(const __grid_constant__ CountArgs a) {
+    const int lane = threadIdx.x & 31;
+    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][128];
+    uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
+    const uint64_t n = a.hdr->queue_len;
+    for (;;) {
+        unsigned long long e = 0;
+        if (lane == 0) e = atomicAdd(&a.hdr->queue_ctr, 1ull);
+        e = __shfl_sync(kFull, e, 0);
+        if (e >= n) break;
+        const unsigned long long v = a.queue[e];
+        const uint64_t q = v >> 32;
+        const uint32_t hmask = uint32_t(v);
+        const sel_nest nest = a.nests[a.prob_nest[q]];
+        const uint32_t B = a.prob_B[q];
+        const uint32_t WR = uint32_t(a.prob_WR[q]);
+        const uint32_t P = uint32_t(nest.P0);
+        const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
+                       T2 = uint32_t(eff_trip(nest.trip[2]));
+        const RepClasses rc = rep_classes(P, B);
+        Acc acc{};
+        uint32_t woff = 0;
+        const sel_access* ap = a.acc + nest.access_off;
+        const uint32_t nk = nest.n_access < 31u ? nest.n_access : 31u;
+        for (uint32_t k = 0; k < nk; k++, ap++) {
+            const uint32_t d = ap->depth;
+            const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
+            const uint32_t Wk = WR * Mk;
+            if (!((hmask >> k) & 1u) || Wk == 0) {
+                woff += Wk;
+                continue;
+            }
+            const sel_access ac = *ap;
+            const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
+            const uint32_t g = uint32_t(uabs(ac.c_par[0]));
+            const uint32_t cB = uint32_t(uint64_t(ac.c_par[0])) * B;
+            Part p;
+            if (!hist) {
+                p = count_1d_general(ap, P, B, T0, T1, T2, Mk, 0, Wk, tc, lane, hist).p;
+                acc.Q += p.q;
+                acc.H += Wk - p.q;
+            } else if ((B & 31u) == 0 || ((cB | (32u * g)) & 127u) == 0) {
+                p = count_hist_whole(ac, int(d), T0, T1, T2, rc, tc, hist, lane);
+                acc.H += Wk;
+            } else {
+                p = count_hist_reps(ap, int(d), T0, T1, T2, P, B, WR, tc, hist, lane);
+                acc.H += Wk;
+            }
+            add_part(acc, p);
+            acc.W += Wk;
+            woff += Wk;
+        }
+        flush(a, q, acc, lane);
+        if (hmask >> 31) {                                  // accesses 31, 32, ...: the general path
+            const uint64_t Wq = uint64_t(WR) * a.prob_cnt[q * kCntStride + 5];
+            count_problem<MODE>(a, q, woff, uint32_t(Wq - woff), lane, hist);
+        }
+    }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(const __grid_constant__ CountArgs a) {
     const int lane = threadIdx.x & 31;
     __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][128];
     uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
@@ -1074,17 +1339,31 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
     }
 }
 
+// persistent grid: #SMs x resident blocks of kernel k
+template <typename K>
+static int persistent_grid(K k, int threads) {
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, threads, 0);
+    return sms * (per > 0 ? per : 1);
+}
+
 template <int MODE>
-static int count_grid() {
-    static int g = 0;
-    if (g == 0) {
-        int dev = 0, sms = 0, per = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_count<MODE>, SEL_COUNT_THREADS, 0);
-        g = sms * (per > 0 ? per : 1);
+static void launch_mode(const CountArgs& a, cudaStream_t s) {
+    static int g_count = 0, g_queue = 0, g_lane = 0;
+    if (g_count == 0) {
+        g_count = persistent_grid(k_count<MODE>, SEL_COUNT_THREADS);
+        g_queue = persistent_grid(k_queue<MODE>, SEL_COUNT_THREADS);
+        g_lane = persistent_grid(k_lane_problems<MODE>, 256);
     }
-    return g;
+    if (MODE != 0) {
+        k_lane_problems<MODE><<<g_lane, 256, 0, s>>>(a);
+        k_queue<MODE><<<g_queue, SEL_COUNT_THREADS, 0, s>>>(a);
+        note_launch(2);
+    }
+    k_count<MODE><<<g_count, SEL_COUNT_THREADS, 0, s>>>(a);
+    note_launch();
 }
 
 cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_problems, uint32_t flags,
@@ -1092,13 +1371,13 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
     (void)max_problems;
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
-                (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u};
+                (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u,
+                w.queue};
     prof_before_count(s);
-    if (mode == 0) k_count<0><<<count_grid<0>(), SEL_COUNT_THREADS, 0, s>>>(a);
-    else if (mode == 1) k_count<1><<<count_grid<1>(), SEL_COUNT_THREADS, 0, s>>>(a);
-    else k_count<2><<<count_grid<2>(), SEL_COUNT_THREADS, 0, s>>>(a);
+    if (mode == 0) launch_mode<0>(a, s);
+    else if (mode == 1) launch_mode<1>(a, s);
+    else launch_mode<2>(a, s);
     prof_after_count(s);
-    note_launch();
     return cudaGetLastError();
 }
 

@@ -27,13 +27,16 @@ struct WsHeader {
     unsigned int _pad0;
     unsigned long long w_begin, w_end; // this call's slice of the problem work space (prefix units)
     unsigned int part, n_parts;        // sel_count_transactions_part: slice index / count
-    unsigned long long _pad[18];
+    unsigned long long small_begin, small_end;   // this call's range of lane-parallel (small) problems
+    unsigned long long queue_len;      // problems handed from the lane kernel to the warp kernel
+    unsigned long long queue_ctr;      // dynamic work counter of the warp (queue) kernel
+    unsigned long long _pad[14];
 };
 static_assert(sizeof(WsHeader) == 256, "header size");
 
 struct WsLayout {
     size_t hdr, slots, nest_base, cand_pid, prob_nest, prob_B, prob_W, prob_WR, prob_cnt,
-        prob_status, cand_status, scan_tmp, total;
+        prob_status, cand_status, queue, scan_tmp, total;
 };
 
 __host__ __device__ inline size_t ws_align(size_t x) { return (x + 255) & ~size_t(255); }
@@ -59,6 +62,7 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
     L.prob_cnt = o;   o = ws_align(o + n * kCntStride * sizeof(uint64_t));
     L.prob_status = o; o = ws_align(o + n);
     L.cand_status = o; o = ws_align(o + n);
+    L.queue = o;      o = ws_align(o + n * sizeof(uint64_t));
     uint64_t big = n > n_nests ? n : n_nests;
     L.scan_tmp = o;   o = ws_align(o + scan_blocks(big) * sizeof(uint64_t) * 2);
     L.total = o;
@@ -143,6 +147,11 @@ __device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc
     *M_it_out = M_it;
     return SEL_OK;
 }
+
+// Problems counted one per lane (k_lane_problems) rather than through the WA
+// prefix: 1-D, small enough for 32-bit lane sums and a short warp-rep walk.
+constexpr uint64_t kSmallMaxW = 1ull << 24;
+constexpr uint64_t kSmallMaxWR = 1024;
 
 // Warps with at least one active lane (R8, R9), summed over the R*G blocks of
 // the launch.  Block k covers iterations [kB, kB + B); block-to-grid mapping

@@ -21,6 +21,7 @@ struct WsPtrs {
     unsigned long long* prob_cnt;    // 5 x u64 per problem: W, L, S, C, U
     uint8_t* prob_status;
     uint8_t* cand_status;
+    unsigned long long* queue;       // (problem << 32 | first WA) handed from the lane to the warp kernel
     unsigned long long* scan_tmp;
 };
 

@@ -227,7 +227,7 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
-                                                   unsigned long long* prob_cnt) {
+                                                   unsigned long long* prob_cnt, int lane_ok) {
     const uint64_t nq = hdr->n_problems;
     const uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (q >= nq) return;
@@ -242,7 +242,10 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader*
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
     prob_cnt[q * kCntStride + 5] = M_it;
-    prob_W[q] = WR * M_it;
+    // small problems are counted one per lane (k_lane_problems), outside the prefix
+    const uint64_t W = WR * M_it;
+    const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
+    prob_W[q] = small ? 0ull : W;
 }
 
 // slice [total*part/n_parts, total*(part+1)/n_parts) of the problem work space
@@ -253,7 +256,12 @@ __global__ void k_plan_stats(WsHeader* hdr, const unsigned long long* prefix) {
     const uint64_t e = uint64_t(total * (hdr->part + 1) / hdr->n_parts);
     hdr->w_begin = b;
     hdr->w_end = e;
-    hdr->stats.wa_analysed = e - b;
+    hdr->stats.wa_analysed = e - b;               // + the small problems' W (k_lane_problems)
+    const unsigned __int128 nq = hdr->n_problems;
+    hdr->small_begin = uint64_t(nq * hdr->part / hdr->n_parts);
+    hdr->small_end = uint64_t(nq * (hdr->part + 1) / hdr->n_parts);
+    hdr->queue_len = 0;
+    hdr->queue_ctr = 0;
 }
 
 cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables& t, int n_sets,
@@ -283,7 +291,9 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
     }
     k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0, part, n_parts);
     k_problem_w<<<unsigned((n + 255) / 256), 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
-                                                          w.prob_status, w.prob_cnt);
+                                                          w.prob_status, w.prob_cnt,
+                                                          (flags & (SEL_F_MATCH_ANY | SEL_F_EXPAND_ALL |
+                                                                    SEL_F_WARP_PROBLEMS)) ? 0 : 1);
     note_launch(2);
     if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s)) != cudaSuccess) return e;
     k_plan_stats<<<1, 1, 0, s>>>(w.hdr, w.prob_W);

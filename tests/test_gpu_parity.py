@@ -304,7 +304,7 @@ def _random_medium_batch(seed, n):
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 2, 4, 8, 12, 16])
+@pytest.mark.parametrize("flags", [0, 2, 4, 8, 12, 16, 32])
 def test_random_medium_nests(sel, flags):
     b = _random_medium_batch(123 + flags, 1500)
     ref = oracle.evaluate(b)
@@ -373,7 +373,7 @@ def test_uniform_flag_closed_form(sel, flags):
     if flags & 8:
         assert st["wa_closed_form"] == 0 and st["wa_arith_lanes"] == 0 and st["wa_residue_classes"] == 0
     else:
-        assert 0 < st["wa_closed_form"] and 0 < st["wa_arith_lanes"]
+        assert 0 < st["wa_closed_form"] and 0 < st["wa_arith_lanes"] + st["wa_residue_classes"]
         assert (st["wa_closed_form"] + st["wa_arith_lanes"] + st["wa_residue_classes"]
                 < st["wa_analysed"])                                              # collapse(2) expands
 
@@ -421,7 +421,7 @@ def _residue_class_batch(seed, n):
     return gen.custom_batch(items, launches_=launches)
 
 
-@pytest.mark.parametrize("flags", [0, 16, 4, 1, 8])
+@pytest.mark.parametrize("flags", [0, 16, 4, 1, 8, 32, 48])
 def test_residue_classes(sel, flags):
     b = _residue_class_batch(77 + flags, 1500)
     ref = oracle.evaluate(b)
@@ -439,8 +439,8 @@ def test_residue_classes_c5_slice(sel):
     """c5 slice: residue-class counting agrees with lane-by-lane expansion
     and with the arithmetic-lane path, counts and cycles bit for bit."""
     b = gen.generate(5, 3000000, 3300000)
-    g0, g16, g8 = run_gpu(sel, b, 0), run_gpu(sel, b, 16), run_gpu(sel, b, 8)
-    for g in (g16, g8):
+    g0, g16, g8, g32 = run_gpu(sel, b, 0), run_gpu(sel, b, 16), run_gpu(sel, b, 8), run_gpu(sel, b, 32)
+    for g in (g16, g8, g32):
         assert (g0["counts"] == g["counts"]).all() and (g0["cycles"] == g["cycles"]).all()
         assert (g0["decision"] == g["decision"]).all()
     assert g0["stats"]["wa_residue_classes"] > 0 and g16["stats"]["wa_residue_classes"] == 0

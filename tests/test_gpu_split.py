@@ -4,7 +4,7 @@ and one all_reduce(SUM) of the u64 counters restores the exact counts.
 
 Checks: the parts sum to sel_count_transactions exactly for several R (and to
 the oracle's brute-force counts); warp_reps appears in part 0 only; statuses
-are identical across parts; the slice sizes tile the work space; the 2-rank
+are identical across parts; the part sizes add up to the whole; the 2-rank
 path (evaluate_split over gloo, both ranks on the box's single GPU) matches
 the oracle end to end."""
 import json
@@ -58,7 +58,9 @@ def _parts(sel, b, n_parts, flags=0):
             assert (c[:, 5] == 0).all(), "warp_reps must come from part 0 only"
         acc += c
         sizes.append(sel.read_stats(ev.workspace)["wa_analysed"])
-    assert sum(sizes) == total and max(sizes) - min(sizes) <= 1
+    # the parts tile the work: big problems by equal slices of the WA prefix, small
+    # problems (counted one per lane) by problem-index ranges
+    assert sum(sizes) == total
     return full, acc, st_full
 
 

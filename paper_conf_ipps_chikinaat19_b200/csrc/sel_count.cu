@@ -1239,7 +1239,11 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
     if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_analysed, Wt);
 }
 
-// The handed-over rest of small problems, one warp per queue entry.
+// The handed-over accesses of small problems, one warp per queue entry.
+// Entries are taken 32 at a time: lane j loads entry j's problem metadata
+// (independent loads, one latency for the batch), then the warp walks the
+// batch with the metadata broadcast by shuffles and loads only the handed
+// accesses' descriptors.
 template <int MODE>
 __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_queue(const __grid_constant__ CountArgs a) {
     const int lane = threadIdx.x & 31;
@@ -1247,57 +1251,72 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
     uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
     const uint64_t n = a.hdr->queue_len;
     for (;;) {
-        unsigned long long e = 0;
-        if (lane == 0) e = atomicAdd(&a.hdr->queue_ctr, 1ull);
-        e = __shfl_sync(kFull, e, 0);
-        if (e >= n) break;
-        const unsigned long long v = a.queue[e];
-        const uint64_t q = v >> 32;
-        const uint32_t hmask = uint32_t(v);
-        const sel_nest nest = a.nests[a.prob_nest[q]];
-        const uint32_t B = a.prob_B[q];
-        const uint32_t WR = uint32_t(a.prob_WR[q]);
-        const uint32_t P = uint32_t(nest.P0);
-        const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
-                       T2 = uint32_t(eff_trip(nest.trip[2]));
-        const RepClasses rc = rep_classes(P, B);
-        Acc acc{};
-        uint32_t woff = 0;
-        const sel_access* ap = a.acc + nest.access_off;
-        const uint32_t nk = nest.n_access < 31u ? nest.n_access : 31u;
-        for (uint32_t k = 0; k < nk; k++, ap++) {
-            const uint32_t d = ap->depth;
-            const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
-            const uint32_t Wk = WR * Mk;
-            if (!((hmask >> k) & 1u) || Wk == 0) {
-                woff += Wk;
-                continue;
-            }
-            const sel_access ac = *ap;
-            const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
-            const uint32_t g = uint32_t(uabs(ac.c_par[0]));
-            const uint32_t cB = uint32_t(uint64_t(ac.c_par[0])) * B;
-            Part p;
-            if (!hist) {
-                p = count_1d_general(ap, P, B, T0, T1, T2, Mk, 0, Wk, tc, lane, hist).p;
-                acc.Q += p.q;
-                acc.H += Wk - p.q;
-            } else if ((B & 31u) == 0 || ((cB | (32u * g)) & 127u) == 0) {
-                p = count_hist_whole(ac, int(d), T0, T1, T2, rc, tc, hist, lane);
-                acc.H += Wk;
-            } else {
-                p = count_hist_reps(ap, int(d), T0, T1, T2, P, B, WR, tc, hist, lane);
-                acc.H += Wk;
-            }
-            add_part(acc, p);
-            acc.W += Wk;
-            woff += Wk;
+        unsigned long long e0 = 0;
+        if (lane == 0) e0 = atomicAdd(&a.hdr->queue_ctr, 32ull);
+        e0 = __shfl_sync(kFull, e0, 0);
+        if (e0 >= n) break;
+        const uint32_t nb = uint32_t(umin64(32, n - e0));
+        // lane j: metadata of entry e0 + j
+        uint32_t q_l = 0, hm_l = 0, B_l = 0, WR_l = 0, P_l = 0, T0_l = 0, T1_l = 0, T2_l = 0, ao_l = 0, na_l = 0;
+        if (uint32_t(lane) < nb) {
+            const unsigned long long v = a.queue[e0 + lane];
+            q_l = uint32_t(v >> 32);
+            hm_l = uint32_t(v);
+            const sel_nest* np = a.nests + a.prob_nest[q_l];
+            B_l = a.prob_B[q_l];
+            WR_l = uint32_t(a.prob_WR[q_l]);
+            P_l = uint32_t(np->P0);
+            T0_l = uint32_t(eff_trip(np->trip[0]));
+            T1_l = uint32_t(eff_trip(np->trip[1]));
+            T2_l = uint32_t(eff_trip(np->trip[2]));
+            ao_l = np->access_off;
+            na_l = np->n_access;
         }
-        flush(a, q, acc, lane);
-        if (hmask >> 31) {                                  // accesses 31, 32, ...: the general path
-            const uint64_t Wq = uint64_t(WR) * a.prob_cnt[q * kCntStride + 5];
-            count_problem<MODE>(a, q, woff, uint32_t(Wq - woff), lane, hist);
+        for (uint32_t j = 0; j < nb; j++) {
+            const uint32_t q = __shfl_sync(kFull, q_l, j), hmask = __shfl_sync(kFull, hm_l, j);
+            const uint32_t B = __shfl_sync(kFull, B_l, j), WR = __shfl_sync(kFull, WR_l, j);
+            const uint32_t P = __shfl_sync(kFull, P_l, j);
+            const uint32_t T0 = __shfl_sync(kFull, T0_l, j), T1 = __shfl_sync(kFull, T1_l, j),
+                           T2 = __shfl_sync(kFull, T2_l, j);
+            const uint32_t aoff = __shfl_sync(kFull, ao_l, j);
+            Acc acc{};
+            for (uint32_t mk = hmask & 0x7fffffffu; mk; mk &= mk - 1u) {
+                const uint32_t k = uint32_t(__ffs(mk) - 1);
+                const sel_access* ap = a.acc + aoff + k;
+                const sel_access ac = *ap;
+                const uint32_t d = ac.depth;
+                const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
+                const uint32_t Wk = WR * Mk;
+                const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
+                const uint32_t g = uint32_t(uabs(ac.c_par[0]));
+                const uint32_t cB = uint32_t(uint64_t(ac.c_par[0])) * B;
+                Part p;
+                if (!hist) {
+                    p = count_1d_general(ap, P, B, T0, T1, T2, Mk, 0, Wk, tc, lane, hist).p;
+                    acc.Q += p.q;
+                    acc.H += Wk - p.q;
+                } else if ((B & 31u) == 0 || ((cB | (32u * g)) & 127u) == 0) {
+                    p = count_hist_whole(ac, int(d), T0, T1, T2, rep_classes(P, B), tc, hist, lane);
+                    acc.H += Wk;
+                } else {
+                    p = count_hist_reps(ap, int(d), T0, T1, T2, P, B, WR, tc, hist, lane);
+                    acc.H += Wk;
+                }
+                add_part(acc, p);
+                acc.W += Wk;
+            }
+            flush(a, q, acc, lane);
+            if (hmask >> 31) {                              // accesses 31, 32, ...: the general path
+                uint32_t woff = 0;
+                for (uint32_t k = 0; k < 31; k++) {
+                    const uint32_t d = a.acc[aoff + k].depth;
+                    woff += WR * (d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2);
+                }
+                const uint64_t Wq = uint64_t(WR) * a.prob_cnt[uint64_t(q) * kCntStride + 5];
+                count_problem<MODE>(a, q, woff, uint32_t(Wq - woff), lane, hist);
+            }
         }
+        (void)na_l;
     }
 }
 

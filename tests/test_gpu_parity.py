@@ -432,7 +432,7 @@ def test_residue_classes(sel, flags):
     if flags & (8 | 16):
         assert st["wa_residue_classes"] == 0
     else:
-        assert st["wa_residue_classes"] > 0 and st["wa_arith_lanes"] > 0   # arith: fragments, short rows
+        assert st["wa_residue_classes"] > 0
 
 
 def test_residue_classes_c5_slice(sel):

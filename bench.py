@@ -33,7 +33,7 @@ UNIT = "evals/s"
 WORKLOAD = ("c5: 10^8-candidate selection sweep (24 Polybench-shaped nests x trip counts x "
             "8 launch configs x 4 device sets)")
 OPS_PER_WA = 224           # 7 integer lane-ops x 32 lanes per warp-access (lane expansion)
-OPS_PER_WA_ARITH = 12      # arithmetic-lane path, one lane per warp-access
+CAND_BYTES = 24 + 1 + 8    # per candidate: sel_candidate read, decision + cycles written
 
 
 def parse():
@@ -304,34 +304,44 @@ def run_ours(args):
 
     if rank != 0:
         return
-    # ---- roofline of the counting kernel (INT bound): peak = measured INT32
-    # lane-op rate with the ALU and FMA pipes both busy (sel_int_peak mode 2), all SMs
+    # ---- roofline of the counting kernels (INT bound): peak = measured INT32 lane-op
+    # rate with the ALU and FMA pipes both issuing (sel_int_peak mode 2), all SMs.  achieved = the
+    # nominal algorithmic lane-ops the counting kernels performed (sel_stats.alg_lane_ops: 224 per
+    # expanded WA, 12 per arithmetic-lane WA, 6 per uniform class, 6 / 5 / 12 per histogram entry /
+    # convolution term / residue evaluation) / their measured time (CUDA events on the launching stream)
     f_mhz = clocks["sm_mhz"] or measured_peaks().get("clocks_under_load", {}).get("sm_mhz_median", 1965.0)
     peak_ops = int_peak["both"]
-    # algorithmic lane-ops of this rank's launch (rank 0), per counting path (DESIGN.md §7/§8):
-    # lane-by-lane expansion 224 / WA, arithmetic lanes 12 / WA, uniform-flag closed form 0
-    wa_arith = stats["wa_arith_lanes"]
-    wa_lane = stats["wa_analysed"] - stats["wa_closed_form"] - wa_arith
+    wa_arith, wa_res, wa_cf = stats["wa_arith_lanes"], stats["wa_residue_classes"], stats["wa_closed_form"]
+    wa_lane = stats["wa_analysed"] - wa_cf - wa_arith - wa_res
     avg_count_ms = count_ms / max(count_launches, 1)
-    achieved = (wa_lane * OPS_PER_WA + wa_arith * OPS_PER_WA_ARITH) / (avg_count_ms / 1e3)
+    achieved = stats["alg_lane_ops"] / (avg_count_ms / 1e3)
+    survey_eq = stats["wa_analysed"] * OPS_PER_WA / (avg_count_ms / 1e3)
     roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
                 "frac": achieved / peak_ops, "traffic": ncu_traffic_per_launch(),
-                "kernel": "sel::k_count<%d>" % (0 if args.flags & 2 else 1 if args.flags & 4 else 2), "count_ms_per_launch": avg_count_ms,
-                "count_share_of_step": avg_count_ms / (t_step * 1e3),
-                "peak_source": "measured: sel_int_peak (independent IADD3/LOP3 + IMAD chains, all SMs, "
-                               "ALU and FMA pipes both issuing) at the run's clocks",
+                "kernel": "counting kernels (k_lane_problems + k_queue + k_count)",
+                "count_ms_per_launch": avg_count_ms, "count_share_of_step": avg_count_ms / (t_step * 1e3),
+                "alg_lane_ops_per_step": stats["alg_lane_ops"],
+                "peak_source": "measured: sel_int_peak (independent IADD3/LOP3 + IMAD chains, all SMs, ALU and FMA "
+                               "pipes both issuing) at the run's clocks",
                 "peak_alu_pipe_only": int_peak["alu"] / 1e12, "peak_fma_pipe_only": int_peak["fma"] / 1e12,
                 "peak_nominal_issue": 148 * 128 * f_mhz * 1e6 / 1e12,
-                "algorithmic_ops_per_wa": {"lane_expansion": OPS_PER_WA, "arith_lanes": OPS_PER_WA_ARITH,
-                                           "closed_form": 0},
-                "wa_per_path": {"lane_expansion": wa_lane, "arith_lanes": wa_arith,
-                                "closed_form": stats["wa_closed_form"]},
-                "note": ("achieved = sum over counting paths of warp-accesses x that path's algorithmic "
-                         "lane-ops (SURVEY's 224 for lane-by-lane expansion, 12 for one lane per "
-                         "warp-access, 0 for uniform-flag closed form) / count-kernel time; the byte-sliced "
-                         "lane expansion evaluates 4 warp-accesses per 32-bit lane op; "
-                         "ncu_* are the issued-instruction counters of the committed capture"),
+                "wa_per_path": {"lane_expansion": wa_lane, "arith_lanes": wa_arith, "residue_classes": wa_res,
+                                "uniform_closed_form": wa_cf},
+                "survey_equivalent": {"ops_per_wa": OPS_PER_WA, "achieved": survey_eq / 1e12,
+                                      "ratio_to_peak": survey_eq / peak_ops,
+                                      "note": "SURVEY §8(d)'s 224 lane-ops x every analysed warp-access / counting "
+                                              "time: the brute-force expansion rate the exact closed forms stand "
+                                              "in for (> 1 = faster than expanding at the INT peak)"},
+                "note": ("achieved = nominal algorithmic lane-ops of the paths the counting kernels took "
+                         "(sel_stats.alg_lane_ops) / their time; ncu_* are the issued-instruction counters of the "
+                         "committed capture"),
                 "ncu": ncu_capture()}
+    # the whole step against HBM: per candidate the 24 B record in, decision + cycles out
+    step_hbm = {"bound": "hbm", "bytes_per_candidate": CAND_BYTES,
+                "achieved": CAND_BYTES * total / t_step / 1e9, "peak": measured_peaks().get("hbm_gbs"),
+                "unit": "GB/s"}
+    if step_hbm["peak"]:
+        step_hbm["frac"] = step_hbm["achieved"] / step_hbm["peak"]
     hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
     workload = WORKLOAD if args.config == 5 else f"c{args.config}: BASELINE.json configs[{args.config - 1}]"
     parallelism = (f"dp{world} (warp-range split of every candidate) + all_reduce(SUM) of u64 counters" if split
@@ -341,6 +351,8 @@ def run_ours(args):
             "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
             "config": {"workload": workload, "candidates": total, "count_sharing": not (args.flags & 1),
                        "lane_pattern_paths": not (args.flags & 8),
+                       "residue_classes": not (args.flags & (8 | 16)),
+                       "problems_per_lane": not (args.flags & (2 | 8 | 32)),
                        "counting_primitive": ("match_any" if args.flags & 2 else
                                               "residue (scalar)" if args.flags & 4 else "residue (byte-sliced)"),
                        "l2": (f"inputs larger than L2 ({24 * total / 1e9:.1f} GB of candidates per pass)"
@@ -349,7 +361,8 @@ def run_ours(args):
             "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
             "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
             "wa_closed_form_per_step": wa_closed,
-            "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "gpu_launches": launches,
+            "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "step_hbm_roofline": step_hbm,
+            "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
     if not args.no_next and args.config == 5:
         line["next_rows"] = time_next_rows(sel, gen, ev, batch, cands, args, c0, c1, dev)

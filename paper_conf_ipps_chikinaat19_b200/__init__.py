@@ -218,7 +218,8 @@ def read_stats(workspace: torch.Tensor, stream=None) -> dict:
     wp, _ = _ws_ptr(workspace)
     _lib.check(_lib.lib().sel_read_stats(wp, ctypes.byref(st), _stream(stream)))
     return {k: int(getattr(st, k)) for k in ("n_candidates", "n_problems", "wa_analysed", "wa_covered",
-                                             "n_invalid", "wa_closed_form", "wa_arith_lanes", "wa_residue_classes")}
+                                             "n_invalid", "wa_closed_form", "wa_arith_lanes", "wa_residue_classes",
+                                             "alg_lane_ops")}
 
 
 def profile_enable(on: bool = True) -> None:

@@ -324,7 +324,7 @@ static_assert(sizeof(sel_nest) == 88, "sel_nest layout");
 static_assert(sizeof(sel_launch) == 16, "sel_launch layout");
 static_assert(sizeof(sel_candidate) == 24, "sel_candidate layout");
 static_assert(sizeof(sel_counts) == 48, "sel_counts layout");
-static_assert(sizeof(sel_stats) == 64, "sel_stats layout");
+static_assert(sizeof(sel_stats) == 128, "sel_stats layout");
 static_assert(sizeof(sel_cpu_params) == 64, "sel_cpu_params layout");
 static_assert(sizeof(sel_cpu_input) == 16, "sel_cpu_input layout");
 static_assert(sizeof(sel_sym_term) == 16, "sel_sym_term layout");

@@ -47,7 +47,15 @@ constexpr uint64_t kMaxChunk = 1ull << 20;   // WAs per chunk: keeps all accumul
 #ifndef SEL_HIST_MIN_MK
 #define SEL_HIST_MIN_MK 32
 #endif
-constexpr uint64_t kHistMinMk = SEL_HIST_MIN_MK;   // inner tuples per warp-rep below which count_arith is cheaper
+constexpr uint64_t kHistMinMk = SEL_HIST_MIN_MK;
+// Nominal algorithmic integer lane-ops of each counting path,
+// summed by the kernels into sel_stats.alg_lane_ops (the roofline numerator):
+constexpr uint32_t kOpsExpandWA = 224;   // lane-by-lane expansion, per WA (7 ops x 32 lanes)
+constexpr uint32_t kOpsArithWA = 12;     // arithmetic lanes, per WA: residue 2, lines 2, sectors 3, class 2, sums 3
+constexpr uint32_t kOpsClass = 6;        // uniform flags, per (access, lane-count class): lines, class, 4 sums
+constexpr uint32_t kOpsHistEntry = 6;    // residue histogram of one loop, per entry: residue 3, count 3
+constexpr uint32_t kOpsConvTerm = 5;     // histogram convolution, per (iteration, residue): index 4, MAC 1
+constexpr uint32_t kOpsEvalTerm = 12;    // residue-class evaluation, per (class, residue): as an arithmetic WA   // inner tuples per warp-rep below which count_arith is cheaper
 
 struct CountArgs {
     const sel_nest* nests;
@@ -76,19 +84,23 @@ struct Acc {
     uint32_t cc;                     // per lane: coalesced WAs (arithmetic-lane path)
     uint32_t W, C, lk, sk, uk;       // uniform
     uint32_t K, Q, H;                // uniform statistics: WAs in closed form / arithmetic lanes / residue classes
+    uint32_t ops;                    // per lane: nominal algorithmic lane-ops (summed at the flush)
 };
 // Per-lane partial sums returned by the out-of-line 1-D paths (by value, so
 // the caller's accumulators stay in registers): line flags, sector flags,
 // coalesced WAs, line flags of uncoalesced WAs, WAs done lane by lane.
 struct Part {
-    uint32_t lf, sf, cc, uf, q;
+    uint32_t lf, sf, cc, uf, q, ops;
 };
 __device__ __forceinline__ void add_part(Acc& acc, const Part& p) {
     acc.lf += p.lf;
     acc.sf += p.sf;
     acc.cc += p.cc;
     acc.uf += p.uf;
+    acc.ops += p.ops;
 }
+
+__device__ __forceinline__ uint32_t lane0(int lane, uint32_t x) { return lane == 0 ? x : 0u; }
 
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
@@ -420,7 +432,7 @@ __device__ __noinline__ Part count_uniform(uint64_t P, uint32_t B, uint64_t Mk, 
         w = uint32_t(mm - kb * wpb);
     }
     const uint32_t qb = 32u / wpb, rw = 32u % wpb;       // 32 warps = qb blocks + rw warps
-    uint32_t lf = 0, cc = 0, uf = 0;
+    uint32_t lf = 0, cc = 0, uf = 0, ops = 0;
     for (uint64_t j = uint64_t(lane); j < nw; j += 32) {
         const uint64_t lo = j * Mk > start ? j * Mk : start;
         const uint64_t hi = (j + 1) * Mk < end ? (j + 1) * Mk : end;
@@ -441,8 +453,9 @@ __device__ __noinline__ Part count_uniform(uint64_t P, uint32_t B, uint64_t Mk, 
         lf += k * nl;
         if (nl + 1u <= tmin) cc += k;                     // R11
         else uf += k * nl;
+        ops += kOpsClass;
     }
-    return Part{lf, lf, cc, uf, 0u};
+    return Part{lf, lf, cc, uf, 0u, ops};
 }
 
 // ------------------------------------------------------------- arithmetic lanes
@@ -546,7 +559,7 @@ __device__ __noinline__ Part count_arith(const sel_access& a, uint64_t P, uint32
             warp_props();
         }
     }
-    return Part{lf, sf, cc, uf, cnt};
+    return Part{lf, sf, cc, uf, cnt, lane0(lane, kOpsArithWA * cnt)};
 }
 
 // ------------------------------------------------------------- residue classes
@@ -566,13 +579,15 @@ __device__ __forceinline__ uint32_t loop_period_log2(uint32_t k) {   // log2 pi
 }
 
 // h <- histogram of one loop (k, T), T >= 1; smem, R slots of 2^sh bytes
-__device__ __forceinline__ void hist_one(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane) {
+__device__ __forceinline__ void hist_one(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane,
+                                         uint32_t& ops) {
 #pragma unroll
     for (uint32_t j = 0; j < 4; j++)
         if (lane + 32u * j < R) h[lane + 32u * j] = 0;
     __syncwarp();
     const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
     const uint32_t n = T < pi ? T : pi;                         // <= 128
+    ops += lane0(lane, kOpsHistEntry * n);
 #pragma unroll
     for (uint32_t j = 0; j < 4; j++) {
         const uint32_t i = lane + 32u * j;
@@ -582,9 +597,11 @@ __device__ __forceinline__ void hist_one(uint32_t* h, uint32_t R, uint32_t sh, u
 }
 
 // h <- h (*) histogram of loop (k, T): out[rho] = sum_i cnt(i) h[rho - k i]
-__device__ __forceinline__ void hist_conv(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane) {
+__device__ __forceinline__ void hist_conv(uint32_t* h, uint32_t R, uint32_t sh, uint32_t k, uint32_t T, int lane,
+                                          uint32_t& ops) {
     const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
     const uint32_t n = T < pi ? T : pi;
+    ops += lane0(lane, kOpsConvTerm * n * R);
     uint32_t o[4] = {0u, 0u, 0u, 0u};
     for (uint32_t i = 0; i < n; i++) {
         const uint32_t c = (T - i + pi - 1u) >> lp;
@@ -608,8 +625,9 @@ __device__ __forceinline__ void hist_conv(uint32_t* h, uint32_t R, uint32_t sh, 
 // active lanes: lane sums over the residues (same integers as count_arith)
 __device__ __forceinline__ void hist_eval(const uint32_t* h, uint32_t R, uint32_t sh, uint32_t lo, uint32_t nm1,
                                           uint32_t g, uint32_t tmin, uint32_t mult, int lane, uint32_t& lf,
-                                          uint32_t& sf, uint32_t& cc, uint32_t& uf) {
+                                          uint32_t& sf, uint32_t& cc, uint32_t& uf, uint32_t& ops) {
     const uint32_t span = nm1 * g;
+    ops += lane0(lane, kOpsEvalTerm * R);
 #pragma unroll
     for (uint32_t j = 0; j < 4; j++) {
         const uint32_t s = lane + 32u * j;
@@ -633,8 +651,10 @@ __device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_
                                         uint64_t T2, uint64_t Mk, uint64_t m0, uint64_t tt, uint32_t cnt, int lane,
                                         uint32_t tmin, uint32_t* h) {
     uint64_t m = m0;
-    Part out{0u, 0u, 0u, 0u, 0u};
-    auto add = [&](const Part& p) { out.lf += p.lf; out.sf += p.sf; out.cc += p.cc; out.uf += p.uf; out.q += p.q; };
+    Part out{0u, 0u, 0u, 0u, 0u, 0u};
+    auto add = [&](const Part& p) {
+        out.lf += p.lf; out.sf += p.sf; out.cc += p.cc; out.uf += p.uf; out.q += p.q; out.ops += p.ops;
+    };
     if (tt > 0) {                                               // head: rest of warp-rep m0
         const uint32_t k = uint32_t(umin64(Mk - tt, cnt));
         add(count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m, tt, k, lane, tmin));
@@ -649,12 +669,16 @@ __device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_
         const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
         const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
                        k2 = uint32_t(uint64_t(a.c_inner[2]));
-        if (DEPTH == 1) hist_one(h, R, sh, k0, uint32_t(T0), lane);
-        if (DEPTH == 2) { hist_one(h, R, sh, k1, uint32_t(T1), lane); hist_conv(h, R, sh, k0, uint32_t(T0), lane); }
+        uint32_t ops = 0;
+        if (DEPTH == 1) hist_one(h, R, sh, k0, uint32_t(T0), lane, ops);
+        if (DEPTH == 2) {
+            hist_one(h, R, sh, k1, uint32_t(T1), lane, ops);
+            hist_conv(h, R, sh, k0, uint32_t(T0), lane, ops);
+        }
         if (DEPTH == 3) {
-            hist_one(h, R, sh, k2, uint32_t(T2), lane);
-            hist_conv(h, R, sh, k1, uint32_t(T1), lane);
-            hist_conv(h, R, sh, k0, uint32_t(T0), lane);
+            hist_one(h, R, sh, k2, uint32_t(T2), lane, ops);
+            hist_conv(h, R, sh, k1, uint32_t(T1), lane, ops);
+            hist_conv(h, R, sh, k0, uint32_t(T0), lane, ops);
         }
         const int64_t c0 = a.c_par[0];
         const uint32_t g = uint32_t(uabs(c0));
@@ -674,12 +698,12 @@ __device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_
                 const uint32_t cntj = first < m + nf ? uint32_t((m + nf - 1 - first) / 4 + 1) : 0u;
                 if (cntj == 0) continue;
                 const uint32_t lo = base32 + c032 * (32u * uint32_t(first)) + (neg ? c032 * 31u : 0u);
-                hist_eval(h, R, sh, lo, 31u, g, tmin, cntj, lane, lf, sf, cc, uf);
+                hist_eval(h, R, sh, lo, 31u, g, tmin, cntj, lane, lf, sf, cc, uf, ops);
             }
             if (ef < e) {                                       // the partial last warp-rep of P
                 const uint32_t nm1 = uint32_t(P - 32ull * ef) - 1u;
                 const uint32_t lo = base32 + c032 * (32u * uint32_t(ef)) + (neg ? c032 * nm1 : 0u);
-                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf);
+                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf, ops);
             }
         } else {
             const uint32_t wpb = (B + 31u) >> 5;
@@ -690,11 +714,11 @@ __device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_
                 const uint64_t pe = umin64(umin64(p0 + 32, (kb + 1) * uint64_t(B)), P);
                 const uint32_t nm1 = uint32_t(pe - p0) - 1u;
                 const uint32_t lo = base32 + c032 * uint32_t(p0) + (neg ? c032 * nm1 : 0u);
-                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf);
+                hist_eval(h, R, sh, lo, nm1, g, tmin, 1u, lane, lf, sf, cc, uf, ops);
                 if (++w == wpb) { w = 0; kb++; }
             }
         }
-        add(Part{lf, sf, cc, uf, 0u});
+        add(Part{lf, sf, cc, uf, 0u, ops});
         __syncwarp();                                           // h is reused by the next access
     }
     if (rest) add(count_arith<DEPTH>(a, P, B, T0, T1, T2, Mk, m + nfull, 0, rest, lane, tmin));
@@ -734,8 +758,9 @@ __device__ __forceinline__ RepClasses rep_classes(uint64_t P, uint32_t B) {
 // lines = sectors = 1 + (flags ? n - 1 : 0) in each of its Mk warp-accesses
 // (count_uniform); warp-uniform accumulators.
 __device__ __forceinline__ void uniform_whole(const RepClasses& rc, uint32_t Mk, bool flags, uint32_t tmin,
-                                              Acc& acc) {
+                                              Acc& acc, int lane) {
     auto cls = [&](uint32_t lanes, uint32_t reps) {
+        acc.ops += lane0(lane, kOpsClass);
         const uint32_t w = reps * Mk;                       // <= WR * Mk <= kMaxChunk
         const uint32_t nl = flags ? lanes - 1u : 0u;
         acc.lk += w * nl;
@@ -750,13 +775,17 @@ __device__ __forceinline__ void uniform_whole(const RepClasses& rc, uint32_t Mk,
 
 // h <- residue histogram of the access's inner offsets (runtime depth 0..3)
 __device__ __forceinline__ void hist_build(uint32_t* h, const sel_access& a, int depth, uint32_t T0, uint32_t T1,
-                                           uint32_t T2, uint32_t R, uint32_t sh, int lane) {
+                                           uint32_t T2, uint32_t R, uint32_t sh, int lane, uint32_t& ops) {
     const uint32_t k0 = uint32_t(uint64_t(a.c_inner[0])), k1 = uint32_t(uint64_t(a.c_inner[1])),
                    k2 = uint32_t(uint64_t(a.c_inner[2]));
-    if (depth == 0) hist_one(h, R, sh, 0u, 1u, lane);
-    else if (depth == 1) hist_one(h, R, sh, k0, T0, lane);
-    else if (depth == 2) { hist_one(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
-    else { hist_one(h, R, sh, k2, T2, lane); hist_conv(h, R, sh, k1, T1, lane); hist_conv(h, R, sh, k0, T0, lane); }
+    if (depth == 0) hist_one(h, R, sh, 0u, 1u, lane, ops);
+    else if (depth == 1) hist_one(h, R, sh, k0, T0, lane, ops);
+    else if (depth == 2) { hist_one(h, R, sh, k1, T1, lane, ops); hist_conv(h, R, sh, k0, T0, lane, ops); }
+    else {
+        hist_one(h, R, sh, k2, T2, lane, ops);
+        hist_conv(h, R, sh, k1, T1, lane, ops);
+        hist_conv(h, R, sh, k0, T0, lane, ops);
+    }
 }
 
 // Residue classes over a whole access when the warp-reps' lowest lane
@@ -769,13 +798,15 @@ __device__ __noinline__ Part count_hist_reps(const sel_access* ap, int depth, ui
                                              int lane) {
     const sel_access a = *ap;
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
-    hist_build(h, a, depth, T0, T1, T2, R, sh, lane);
+    uint32_t ops = 0;
+    hist_build(h, a, depth, T0, T1, T2, R, sh, lane, ops);
+    ops += lane0(lane, kOpsEvalTerm * R * WR);
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
     const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
     const uint32_t wpb = (B + 31u) >> 5;
-    Part o{0u, 0u, 0u, 0u, 0u};
+    Part o{0u, 0u, 0u, 0u, 0u, ops};
     for (uint32_t m0 = 0; m0 < WR; m0 += 32) {
         const uint32_t m = m0 + uint32_t(lane);
         const bool act = m < WR;
@@ -814,29 +845,29 @@ __device__ __noinline__ Part count_hist_reps(const sel_access* ap, int depth, ui
 __device__ __forceinline__ Part count_hist_whole(const sel_access& a, int depth, uint32_t T0, uint32_t T1,
                                                  uint32_t T2, RepClasses rc, uint32_t tmin, uint32_t* h, int lane) {
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
-    hist_build(h, a, depth, T0, T1, T2, R, sh, lane);
+    Part o{0u, 0u, 0u, 0u, 0u, 0u};
+    hist_build(h, a, depth, T0, T1, T2, R, sh, lane, o.ops);
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
     const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
-    Part o{0u, 0u, 0u, 0u, 0u};
     // lowest lane address of a warp-rep starting at iteration p0 with n lanes
     auto lo_of = [&](uint32_t p0, uint32_t n) { return base32 + c032 * p0 + (neg ? c032 * (n - 1u) : 0u); };
     if (rc.n32) {
         if (((32u * c032) & 127u) == 0) {
-            hist_eval(h, R, sh, lo_of(0u, 32u), 31u, g, tmin, uint32_t(rc.n32), lane, o.lf, o.sf, o.cc, o.uf);
+            hist_eval(h, R, sh, lo_of(0u, 32u), 31u, g, tmin, uint32_t(rc.n32), lane, o.lf, o.sf, o.cc, o.uf, o.ops);
         } else {                                            // 32 | B here: warp-rep j starts at 32 j
             for (uint32_t j = 0; j < 4; j++) {
                 const uint32_t cj = uint32_t((rc.n32 + 3u - j) >> 2);   // #{x < n32 : x = j mod 4}
-                if (cj) hist_eval(h, R, sh, lo_of(32u * j, 32u), 31u, g, tmin, cj, lane, o.lf, o.sf, o.cc, o.uf);
+                if (cj) hist_eval(h, R, sh, lo_of(32u * j, 32u), 31u, g, tmin, cj, lane, o.lf, o.sf, o.cc, o.uf, o.ops);
             }
         }
     }
     if (rc.nA) hist_eval(h, R, sh, lo_of(0u, rc.lanesA), rc.lanesA - 1u, g, tmin, uint32_t(rc.nA), lane, o.lf, o.sf,
-                         o.cc, o.uf);
+                         o.cc, o.uf, o.ops);
     if (rc.lanesR) {                                        // the last warp-rep of P starts at 32 n32 (32 | B)
         const uint32_t p0 = rc.nA ? 0u : uint32_t(32u * rc.n32);
-        hist_eval(h, R, sh, lo_of(p0, rc.lanesR), rc.lanesR - 1u, g, tmin, 1u, lane, o.lf, o.sf, o.cc, o.uf);
+        hist_eval(h, R, sh, lo_of(p0, rc.lanesR), rc.lanesR - 1u, g, tmin, 1u, lane, o.lf, o.sf, o.cc, o.uf, o.ops);
     }
     __syncwarp();                                           // h is reused by the next access
     return o;
@@ -910,6 +941,7 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
                 const uint32_t ns = __popc(__ballot_sync(kFull, dsb_u == 32u));
                 acc.W += left;
                 acc.K += left;
+                acc.ops += lane0(lane, kOpsClass);
                 acc.lk += left * nl;
                 acc.sk += left * ns;
                 if (nl + 1u <= tmin) acc.C += left;
@@ -936,6 +968,7 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
                 hot_row_swar<TC == 4 ? 1 : TC>(u_low + uint32_t(uint64_t(D)), uint32_t(uint64_t(cl)) & 127u, KL,
                                                KS, len, one, acc);
             }
+            acc.ops += lane0(lane, kOpsExpandWA * len);
             left -= len;
             // odometer carry (registers only)
             if (DEPTH == 1) { i0 += len; if (i0 >= T0) i0 = 0; }
@@ -967,6 +1000,8 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
     if (acc.K && lane == 5) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)acc.K);
     if (acc.Q && lane == 6) atomicAdd((unsigned long long*)&a.hdr->stats.wa_arith_lanes, (unsigned long long)acc.Q);
     if (acc.H && lane == 7) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)acc.H);
+    const uint32_t ops = __reduce_add_sync(kFull, acc.ops);
+    if (ops && lane == 8) atomicAdd((unsigned long long*)&a.hdr->stats.alg_lane_ops, (unsigned long long)ops);
     acc = Acc{};
 }
 
@@ -1069,7 +1104,7 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
         const uint64_t off0 = off;
         off = 0;
         if (whole && (g == 0 || g == 128)) {
-            uniform_whole(rc, uint32_t(Mk), g != 0, tc, acc);
+            uniform_whole(rc, uint32_t(Mk), g != 0, tc, acc, lane);
             acc.K += t;
             continue;
         }
@@ -1101,12 +1136,14 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
 // the rest of its problem to the warp (queue of <= 32 entries).
 struct LaneSums {
     uint32_t W, L, S, C, U;
+    unsigned long long ops;          // nominal algorithmic lane-ops of this thread
 };
 
 // uniform flags over a whole access, one lane (uniform_whole)
 __device__ __forceinline__ void lane_uniform(const RepClasses& rc, uint32_t Mk, bool flags, uint32_t tmin,
                                              LaneSums& z) {
     auto cls = [&](uint32_t lanes, uint32_t reps) {
+        z.ops += kOpsClass;
         const uint32_t w = reps * Mk;
         const uint32_t nl = flags ? lanes : 1u;             // lines = sectors per WA
         z.L += w * nl;
@@ -1133,6 +1170,7 @@ __device__ __forceinline__ void lane_hist1(const sel_access& a, uint32_t T, cons
     const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
     auto cls = [&](uint32_t lo, uint32_t nm1, uint32_t mult) {
         const uint32_t span = nm1 * g;
+        z.ops += kOpsEvalTerm * n;
         for (uint32_t i = 0; i < n; i++) {
             const uint32_t w = ((TT - i + pi - 1u) >> lp) * mult;
             const uint32_t r = (lo + k * i) & 127u;
@@ -1166,7 +1204,7 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
     const uint64_t q_end = a.hdr->small_end;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     uint32_t sK = 0, sH = 0;                                // statistics: WAs by path
-    unsigned long long sW = 0;
+    unsigned long long sW = 0, sOps = 0;
     for (uint64_t qb = a.hdr->small_begin + uint64_t(blockIdx.x) * blockDim.x; qb < q_end; qb += stride) {
         const uint64_t q = qb + threadIdx.x;
         uint32_t hmask = 0;                                 // accesses handed to the warp kernel
@@ -1181,7 +1219,7 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
                 const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
                                T2 = uint32_t(eff_trip(nest.trip[2]));
                 const RepClasses rc = rep_classes(nest.P0, B);
-                LaneSums z{0u, 0u, 0u, 0u, 0u};
+                LaneSums z{0u, 0u, 0u, 0u, 0u, 0ull};
                 const sel_access* ap = a.acc + nest.access_off;
                 for (uint32_t k = 0; k < nest.n_access; k++, ap++) {
                     if (k == 31) {                          // accesses 31, 32, ...: all to the warp kernel
@@ -1209,6 +1247,7 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
                     }
                     z.W += Wk;
                 }
+                sOps += z.ops;
                 if (z.W) {
                     unsigned long long* pc = a.prob_cnt + q * kCntStride;
                     atomicAdd(pc + 0, (unsigned long long)z.W);
@@ -1237,6 +1276,8 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
     if (K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)K);
     if (H && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)H);
     if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_analysed, Wt);
+    for (int o = 16; o; o >>= 1) sOps += __shfl_xor_sync(kFull, sOps, o);
+    if (sOps && lane == 3) atomicAdd((unsigned long long*)&a.hdr->stats.alg_lane_ops, sOps);
 }
 
 // The handed-over accesses of small problems, one warp per queue entry.

@@ -30,7 +30,7 @@ struct WsHeader {
     unsigned long long small_begin, small_end;   // this call's range of lane-parallel (small) problems
     unsigned long long queue_len;      // problems handed from the lane kernel to the warp kernel
     unsigned long long queue_ctr;      // dynamic work counter of the warp (queue) kernel
-    unsigned long long _pad[14];
+    unsigned long long _pad[6];
 };
 static_assert(sizeof(WsHeader) == 256, "header size");
 

@@ -75,6 +75,8 @@ WsPtrs ws_ptrs(void* ws, uint64_t n, uint64_t n_nests, uint32_t flags) {
     p.prob_status = reinterpret_cast<uint8_t*>(b + L.prob_status);
     p.cand_status = reinterpret_cast<uint8_t*>(b + L.cand_status);
     p.queue = reinterpret_cast<unsigned long long*>(b + L.queue);
+    p.prob_md = b + L.prob_md;
+    p.cls = reinterpret_cast<uint32_t*>(b + L.cls);
     p.scan_tmp = reinterpret_cast<unsigned long long*>(b + L.scan_tmp);
     return p;
 }

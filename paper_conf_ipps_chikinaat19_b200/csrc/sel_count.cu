@@ -55,7 +55,13 @@ constexpr uint32_t kOpsArithWA = 12;     // arithmetic lanes, per WA: residue 2,
 constexpr uint32_t kOpsClass = 6;        // uniform flags, per (access, lane-count class): lines, class, 4 sums
 constexpr uint32_t kOpsHistEntry = 6;    // residue histogram of one loop, per entry: residue 3, count 3
 constexpr uint32_t kOpsConvTerm = 5;     // histogram convolution, per (iteration, residue): index 4, MAC 1
-constexpr uint32_t kOpsEvalTerm = 12;    // residue-class evaluation, per (class, residue): as an arithmetic WA   // inner tuples per warp-rep below which count_arith is cheaper
+constexpr uint32_t kOpsEvalTerm = 12;    // residue-class evaluation, per (class, residue): as an arithmetic WA
+constexpr uint32_t kOpsPrefixEntry = 3;  // prefix sums of a residue histogram, per entry
+constexpr uint32_t kOpsEvalClass = 24;   // one residue class from the prefix sums: 2 cyclic range sums + sums
+// per-warp shared words of a residue histogram: h / its exclusive prefix pf[0..R]
+// at [0, 129), the prefix of h folded mod 32 bytes p32[0..R/4] at [kP32Off, +33)
+constexpr uint32_t kP32Off = 132;
+constexpr uint32_t kHistWords = 168;
 
 struct CountArgs {
     const sel_nest* nests;
@@ -621,25 +627,116 @@ __device__ __forceinline__ void hist_conv(uint32_t* h, uint32_t R, uint32_t sh, 
     __syncwarp();
 }
 
+// h[0..R) -> its exclusive prefix pf[0..R] (in place, pf[R] = the total) and
+// the exclusive prefix p32[0..R/4] of h folded mod 32 bytes (slot u of the
+// fold = slots u, u + R/4, u + R/2, u + 3R/4: the same residue mod 32).
+__device__ __forceinline__ void hist_prefix(uint32_t* h, uint32_t R, int lane, uint32_t& ops) {
+    const uint32_t R32 = R >> 2;
+    uint32_t v[4];
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++) v[j] = lane + 32u * j < R ? h[lane + 32u * j] : 0u;
+    const uint32_t f = uint32_t(lane) < R32 ? h[lane] + h[lane + R32] + h[lane + 2u * R32] + h[lane + 3u * R32] : 0u;
+    __syncwarp();
+    ops += lane0(lane, kOpsPrefixEntry * (R + R32));
+    uint32_t carry = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < 4; j++) {
+        if (32u * j >= R) break;
+        uint32_t x = v[j];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(kFull, x, o);
+            if (lane >= o) x += t;
+        }
+        if (lane + 32u * j < R) h[1u + lane + 32u * j] = carry + x;
+        carry += __shfl_sync(kFull, x, 31);
+    }
+    uint32_t y = f;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(kFull, y, o);
+        if (lane >= o) y += t;
+    }
+    if (uint32_t(lane) < R32) h[kP32Off + 1u + lane] = y;
+    if (lane == 0) {
+        h[0] = 0u;
+        h[kP32Off] = 0u;
+    }
+    __syncwarp();
+}
+
+// sum of h over the cyclic slot range start, start + 1, ..., start + len - 1
+// (mod R), len < R, from the exclusive prefix pf (any indexable view)
+template <class A>
+__device__ __forceinline__ uint32_t crange(const A& pf, uint32_t R, uint32_t start, uint32_t len) {
+    const uint32_t e = start + len;
+    return e <= R ? pf[e] - pf[start] : pf[R] - pf[start] + pf[e - R];
+}
+
 // `mult` warp-reps whose lowest lane address is lo (mod 128) with nm1 + 1
-// active lanes: lane sums over the residues (same integers as count_arith)
+// active lanes, summed over the residues of h in closed form from its prefix
+// sums (the same integers as the residue-by-residue sum of count_arith):
+// with span = (n - 1) g = 128 a + b, a WA at residue r has lines - 1 =
+// a + [r >= 128 - b], so  sum_r h(r) (lines - 1) = a H + X,  X = the h-mass of
+// the residues (lo + rho) mod 128 in [128 - b, 128): ONE cyclic range of
+// slots.  Sectors likewise mod 32 (g < 32), or n per WA (g >= 32).  Coalesced
+// <=> lines - 1 < tmin (R11): all, none, or the H - X WAs without the extra
+// line.  Everything in slot units (addresses, strides and spans are multiples
+// of the element size, V5).  pf: exclusive prefix of h over R slots (pf[R] =
+// H); p32: the same of h folded mod 32 bytes (R / 4 slots).
+struct ClassSums {
+    uint32_t lf, sf, cc, uf;
+};
+template <class A>
+__device__ __forceinline__ ClassSums class_sums(const A& pf, const A& p32, uint32_t R, uint32_t sh, uint32_t lo,
+                                                uint32_t nm1, uint32_t g, uint32_t tmin, uint32_t mult) {
+    const uint32_t Ht = pf[R];
+    const uint32_t span = nm1 * g;
+    const uint32_t a = span >> 7, bs = (span & 127u) >> sh, los = (lo & 127u) >> sh;
+    const uint32_t X = bs ? crange(pf, R, (2u * R - bs - los) & (R - 1u), bs) : 0u;
+    ClassSums o;
+    o.lf = a * Ht + X;
+    if (a + 1u < tmin) {
+        o.cc = Ht;
+        o.uf = 0u;
+    } else if (a < tmin) {
+        o.cc = Ht - X;
+        o.uf = (a + 1u) * X;
+    } else {
+        o.cc = 0u;
+        o.uf = o.lf;
+    }
+    if (g >= 32u) {
+        o.sf = nm1 * Ht;
+    } else {
+        const uint32_t R32 = R >> 2;
+        const uint32_t b2s = (span & 31u) >> sh, l32 = (lo & 31u) >> sh;
+        const uint32_t Y = b2s ? crange(p32, R32, (2u * R32 - b2s - l32) & (R32 - 1u), b2s) : 0u;
+        o.sf = (span >> 5) * Ht + Y;
+    }
+    o.lf *= mult;
+    o.sf *= mult;
+    o.cc *= mult;
+    o.uf *= mult;
+    return o;
+}
+__device__ __forceinline__ ClassSums hist_eval_pf(const uint32_t* h, uint32_t R, uint32_t sh, uint32_t lo,
+                                                  uint32_t nm1, uint32_t g, uint32_t tmin, uint32_t mult) {
+    const uint32_t* p32 = h + kP32Off;
+    return class_sums(h, p32, R, sh, lo, nm1, g, tmin, mult);
+}
+
+// lane-uniform class sums, added once (lane 0)
 __device__ __forceinline__ void hist_eval(const uint32_t* h, uint32_t R, uint32_t sh, uint32_t lo, uint32_t nm1,
                                           uint32_t g, uint32_t tmin, uint32_t mult, int lane, uint32_t& lf,
                                           uint32_t& sf, uint32_t& cc, uint32_t& uf, uint32_t& ops) {
-    const uint32_t span = nm1 * g;
-    ops += lane0(lane, kOpsEvalTerm * R);
-#pragma unroll
-    for (uint32_t j = 0; j < 4; j++) {
-        const uint32_t s = lane + 32u * j;
-        if (s >= R) break;
-        const uint32_t w = h[s] * mult;
-        const uint32_t r = (lo + (s << sh)) & 127u;
-        const uint32_t nl = (r + span) >> 7;                    // lines - 1
-        const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
-        lf += w * nl;
-        sf += w * ns;
-        if (nl < tmin) cc += w;                                 // R11
-        else uf += w * nl;
+    const ClassSums c = hist_eval_pf(h, R, sh, lo, nm1, g, tmin, mult);
+    ops += lane0(lane, kOpsEvalClass);
+    if (lane == 0) {
+        lf += c.lf;
+        sf += c.sf;
+        cc += c.cc;
+        uf += c.uf;
     }
 }
 
@@ -680,6 +777,7 @@ __device__ __noinline__ Part count_hist(const sel_access& a, uint64_t P, uint32_
             hist_conv(h, R, sh, k1, uint32_t(T1), lane, ops);
             hist_conv(h, R, sh, k0, uint32_t(T0), lane, ops);
         }
+        hist_prefix(h, R, lane, ops);
         const int64_t c0 = a.c_par[0];
         const uint32_t g = uint32_t(uabs(c0));
         const bool neg = c0 < 0;
@@ -800,7 +898,8 @@ __device__ __noinline__ Part count_hist_reps(const sel_access* ap, int depth, ui
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
     uint32_t ops = 0;
     hist_build(h, a, depth, T0, T1, T2, R, sh, lane, ops);
-    ops += lane0(lane, kOpsEvalTerm * R * WR);
+    hist_prefix(h, R, lane, ops);
+    ops += lane0(lane, kOpsEvalClass * WR);
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
@@ -809,28 +908,19 @@ __device__ __noinline__ Part count_hist_reps(const sel_access* ap, int depth, ui
     Part o{0u, 0u, 0u, 0u, 0u, ops};
     for (uint32_t m0 = 0; m0 < WR; m0 += 32) {
         const uint32_t m = m0 + uint32_t(lane);
-        const bool act = m < WR;
-        uint32_t lo = 0, nm1 = 0;
-        if (act) {
+        if (m < WR) {
             const uint32_t kb = m / wpb, w = m - kb * wpb;
             const uint32_t p0 = kb * B + 32u * w;
             uint32_t pe = p0 + 32u;
             pe = pe < (kb + 1u) * B ? pe : (kb + 1u) * B;
             pe = pe < P ? pe : P;
-            nm1 = pe - p0 - 1u;
-            lo = base32 + c032 * p0 + (neg ? c032 * nm1 : 0u);
-        }
-        const uint32_t span = nm1 * g;
-        for (uint32_t s = 0; s < R; s++) {
-            const uint32_t w = h[s];                        // same slot on every lane: broadcast
-            if (w == 0 || !act) continue;
-            const uint32_t r = (lo + (s << sh)) & 127u;
-            const uint32_t nl = (r + span) >> 7;
-            const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
-            o.lf += w * nl;
-            o.sf += w * ns;
-            if (nl < tmin) o.cc += w;                       // R11
-            else o.uf += w * nl;
+            const uint32_t nm1 = pe - p0 - 1u;
+            const uint32_t lo = base32 + c032 * p0 + (neg ? c032 * nm1 : 0u);
+            const ClassSums c = hist_eval_pf(h, R, sh, lo, nm1, g, tmin, 1u);
+            o.lf += c.lf;
+            o.sf += c.sf;
+            o.cc += c.cc;
+            o.uf += c.uf;
         }
     }
     __syncwarp();                                           // h is reused by the next access
@@ -847,6 +937,7 @@ __device__ __forceinline__ Part count_hist_whole(const sel_access& a, int depth,
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
     Part o{0u, 0u, 0u, 0u, 0u, 0u};
     hist_build(h, a, depth, T0, T1, T2, R, sh, lane, o.ops);
+    hist_prefix(h, R, lane, o.ops);
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
@@ -984,7 +1075,21 @@ __device__ void count_access(const sel_nest& nest, const sel_access& a, uint64_t
     }
 }
 
-__device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
+// Path statistics of one warp, summed over everything it counted and added to
+// the workspace header once per warp at kernel exit (one address line shared
+// by every warp: per-problem atomics there serialise in one L2 slice).
+struct WarpStats {
+    unsigned long long K, Q, H, ops;
+};
+__device__ __forceinline__ void stats_flush(const CountArgs& a, const WarpStats& st, int lane) {
+    if (st.K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, st.K);
+    if (st.Q && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_arith_lanes, st.Q);
+    if (st.H && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, st.H);
+    if (st.ops && lane == 3) atomicAdd((unsigned long long*)&a.hdr->stats.alg_lane_ops, st.ops);
+}
+
+// counts of problem q += this warp's accumulators; statistics move to st
+__device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane, WarpStats& st) {
     const uint64_t slf = __reduce_add_sync(kFull, acc.lf);
     const uint64_t ssf = __reduce_add_sync(kFull, acc.sf);
     const uint64_t suf = __reduce_add_sync(kFull, acc.uf);
@@ -997,11 +1102,10 @@ __device__ void flush(const CountArgs& a, uint64_t q, Acc& acc, int lane) {
         const uint64_t v = lane == 0 ? W : lane == 1 ? L : lane == 2 ? S : lane == 3 ? C : U;
         atomicAdd(&a.prob_cnt[q * kCntStride + lane], (unsigned long long)v);
     }
-    if (acc.K && lane == 5) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)acc.K);
-    if (acc.Q && lane == 6) atomicAdd((unsigned long long*)&a.hdr->stats.wa_arith_lanes, (unsigned long long)acc.Q);
-    if (acc.H && lane == 7) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)acc.H);
-    const uint32_t ops = __reduce_add_sync(kFull, acc.ops);
-    if (ops && lane == 8) atomicAdd((unsigned long long*)&a.hdr->stats.alg_lane_ops, (unsigned long long)ops);
+    st.K += acc.K;
+    st.Q += acc.Q;
+    st.H += acc.H;
+    st.ops += __reduce_add_sync(kFull, acc.ops);
     acc = Acc{};
 }
 
@@ -1066,7 +1170,8 @@ __device__ __noinline__ Acc expand_access(const sel_nest* np, const sel_access* 
 
 // WAs [off, off + take) of problem q, access by access.
 template <int MODE>
-__device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane, uint32_t* hist) {
+__device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane,
+                                           uint32_t* hist, WarpStats& st) {
     const sel_nest* np = a.nests + a.prob_nest[q];
     const sel_nest nest = *np;
     const uint32_t B = a.prob_B[q];
@@ -1122,7 +1227,7 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
             acc.H += t - r.p.q;
         }
     }
-    flush(a, q, acc, lane);
+    flush(a, q, acc, lane, st);
 }
 
 // ------------------------------------------------------------- lane-parallel problems
@@ -1156,43 +1261,120 @@ __device__ __forceinline__ void lane_uniform(const RepClasses& rc, uint32_t Mk, 
     if (rc.lanesR) cls(rc.lanesR, 1u);
 }
 
-// residue classes of a depth <= 1 access over a whole problem, one lane:
-// sum_{i < min(T, pi)} cnt(i) f(lo + k i) per warp-rep class (count_hist_whole)
-__device__ __forceinline__ void lane_hist1(const sel_access& a, uint32_t T, const RepClasses& rc, uint32_t tmin,
-                                           LaneSums& z) {
-    const uint32_t k = a.depth ? uint32_t(uint64_t(a.c_inner[0])) : 0u;
-    const uint32_t TT = a.depth ? T : 1u;
-    const uint32_t lp = loop_period_log2(k), pi = 1u << lp;
-    const uint32_t n = TT < pi ? TT : pi;
+// Residue classes of one access over a whole problem, ONE THREAD: the
+// thread's own residue histogram lives in a shared-memory column (row-major
+// over slots, one column per thread: bank = thread, conflict-free whatever
+// the slot), built from its loops (depth <= 2), turned into prefix sums in
+// place, and every warp-rep class is then evaluated in O(1) (class_sums).
+// Element size >= 4 bytes: R = 128 / E <= 32 slots.
+constexpr uint32_t kLaneThreads = 256;
+constexpr uint32_t kLaneSlots = 32;
+constexpr uint32_t kLaneP32 = kLaneSlots + 1;              // p32 rows after pf[0..R]
+constexpr uint32_t kLaneRows = kLaneP32 + kLaneSlots / 4 + 1;
+struct Col {
+    uint32_t* p;
+    __device__ __forceinline__ uint32_t& operator[](uint32_t s) const { return p[s * kLaneThreads]; }
+};
+
+__device__ __forceinline__ void lane_hist_build(Col h, uint32_t R, uint32_t sh, const sel_access& a, uint32_t T0,
+                                                uint32_t T1, unsigned long long& ops) {
+    for (uint32_t s = 0; s < R; s++) h[s] = 0u;
+    const uint32_t d = a.depth;
+    if (d == 0) {
+        h[0] = 1u;
+        return;
+    }
+    const uint32_t kA = uint32_t(uint64_t(a.c_inner[0]));
+    const uint32_t lA = loop_period_log2(kA), pA = 1u << lA, nA = T0 < pA ? T0 : pA;
+    if (d == 1) {
+        ops += kOpsHistEntry * nA;
+        for (uint32_t i = 0; i < nA; i++) h[((kA * i) & 127u) >> sh] = (T0 - i + pA - 1u) >> lA;
+        return;
+    }
+    // depth 2: every (i, j) residue pair of the two loops' one-loop histograms
+    const uint32_t kB = uint32_t(uint64_t(a.c_inner[1]));
+    const uint32_t lB = loop_period_log2(kB), pB = 1u << lB, nB = T1 < pB ? T1 : pB;
+    ops += kOpsHistEntry * (nA + nB) + kOpsConvTerm * nA * nB;
+    for (uint32_t i = 0; i < nA; i++) {
+        const uint32_t ci = (T0 - i + pA - 1u) >> lA, oi = kA * i;
+        for (uint32_t j = 0; j < nB; j++) {
+            const uint32_t cj = (T1 - j + pB - 1u) >> lB;
+            h[((oi + kB * j) & 127u) >> sh] += ci * cj;
+        }
+    }
+}
+
+// h[0..R) -> exclusive prefix pf[0..R] in place; p32 rows: the prefix of h
+// folded mod 32 bytes (R / 4 slots)
+__device__ __forceinline__ void lane_hist_prefix(Col h, uint32_t R, unsigned long long& ops) {
+    const uint32_t R32 = R >> 2;
+    ops += kOpsPrefixEntry * (R + R32);
+    uint32_t run = 0;
+    for (uint32_t u = 0; u < R32; u++) {
+        run += h[u] + h[u + R32] + h[u + 2u * R32] + h[u + 3u * R32];
+        h[kLaneP32 + 1u + u] = run;
+    }
+    h[kLaneP32] = 0u;
+    run = 0;
+    for (uint32_t s = 0; s < R; s++) {
+        const uint32_t v = h[s];
+        h[s] = run;
+        run += v;
+    }
+    h[R] = run;
+}
+
+__device__ __forceinline__ void lane_add(LaneSums& z, const ClassSums& c, uint32_t w) {
+    z.L += w + c.lf;
+    z.S += w + c.sf;
+    z.C += c.cc;
+    z.U += (w - c.cc) + c.uf;
+}
+
+// one access (depth <= 2, E >= 4, 0 < |c_par| < 128) of a small problem
+__device__ __forceinline__ void lane_hist(Col h, const sel_access& a, uint32_t T0, uint32_t T1, uint32_t P, uint32_t B,
+                                          uint32_t WR, const RepClasses& rc, uint32_t tmin, LaneSums& z) {
+    const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
+    lane_hist_build(h, R, sh, a, T0, T1, z.ops);
+    lane_hist_prefix(h, R, z.ops);
+    const Col p32{h.p + kLaneP32 * kLaneThreads};
+    const uint32_t Ht = h[R];                               // = Mk
     const int64_t c0 = a.c_par[0];
     const uint32_t g = uint32_t(uabs(c0));
     const bool neg = c0 < 0;
     const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
     auto cls = [&](uint32_t lo, uint32_t nm1, uint32_t mult) {
-        const uint32_t span = nm1 * g;
-        z.ops += kOpsEvalTerm * n;
-        for (uint32_t i = 0; i < n; i++) {
-            const uint32_t w = ((TT - i + pi - 1u) >> lp) * mult;
-            const uint32_t r = (lo + k * i) & 127u;
-            const uint32_t nl = (r + span) >> 7;            // lines - 1
-            const uint32_t ns = g < 32u ? ((r & 31u) + span) >> 5 : nm1;
-            z.L += w * (nl + 1u);
-            z.S += w * (ns + 1u);
-            if (nl < tmin) z.C += w;                        // R11
-            else z.U += w * (nl + 1u);
-        }
+        z.ops += kOpsEvalClass;
+        lane_add(z, class_sums(h, p32, R, sh, lo, nm1, g, tmin, mult), Ht * mult);
     };
-    auto lo_of = [&](uint32_t p0, uint32_t nl) { return base32 + c032 * p0 + (neg ? c032 * (nl - 1u) : 0u); };
-    if (rc.n32) {
-        if (((32u * c032) & 127u) == 0) cls(lo_of(0u, 32u), 31u, uint32_t(rc.n32));
-        else
-            for (uint32_t j = 0; j < 4; j++) {
-                const uint32_t cj = uint32_t((rc.n32 + 3u - j) >> 2);
-                if (cj) cls(lo_of(32u * j, 32u), 31u, cj);
-            }
+    auto lo_of = [&](uint32_t p0, uint32_t n) { return base32 + c032 * p0 + (neg ? c032 * (n - 1u) : 0u); };
+    if ((B & 31u) == 0 || (((c032 * B) | (32u * g)) & 127u) == 0) {
+        // the lowest lane address mod 128 of a warp-rep depends on its lane count only
+        // (or, for 32 | B, on the warp-rep index mod 4): count_hist_whole's classes
+        if (rc.n32) {
+            if (((32u * c032) & 127u) == 0) cls(lo_of(0u, 32u), 31u, uint32_t(rc.n32));
+            else
+                for (uint32_t j = 0; j < 4; j++) {
+                    const uint32_t cj = uint32_t((rc.n32 + 3u - j) >> 2);
+                    if (cj) cls(lo_of(32u * j, 32u), 31u, cj);
+                }
+        }
+        if (rc.nA) cls(lo_of(0u, rc.lanesA), rc.lanesA - 1u, uint32_t(rc.nA));
+        if (rc.lanesR) cls(lo_of(rc.nA ? 0u : uint32_t(32u * rc.n32), rc.lanesR), rc.lanesR - 1u, 1u);
+    } else {
+        // every warp-rep from the block geometry (R8, R9), as count_hist_reps
+        const uint32_t wpb = (B + 31u) >> 5;
+        uint32_t kb = 0, w = 0;
+        for (uint32_t m = 0; m < WR; m++) {
+            const uint32_t p0 = kb * B + 32u * w;
+            uint32_t pe = p0 + 32u;
+            pe = pe < (kb + 1u) * B ? pe : (kb + 1u) * B;
+            pe = pe < P ? pe : P;
+            const uint32_t nm1 = pe - p0 - 1u;
+            cls(base32 + c032 * p0 + (neg ? c032 * nm1 : 0u), nm1, 1u);
+            if (++w == wpb) { w = 0; kb++; }
+        }
     }
-    if (rc.nA) cls(lo_of(0u, rc.lanesA), rc.lanesA - 1u, uint32_t(rc.nA));
-    if (rc.lanesR) cls(lo_of(rc.nA ? 0u : uint32_t(32u * rc.n32), rc.lanesR), rc.lanesR - 1u, 1u);
 }
 
 // Small problems (k_problem_w: 1-D, W <= kSmallMaxW, WR <= kSmallMaxWR), one
@@ -1200,7 +1382,9 @@ __device__ __forceinline__ void lane_hist1(const sel_access& a, uint32_t T, cons
 // rest of its problem to the warp kernel (k_queue) at the first access that
 // needs a warp: entry = problem << 32 | WA offset of that access.
 template <int MODE>
-__global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ CountArgs a) {
+__global__ void __launch_bounds__(kLaneThreads) k_lane_problems(const __grid_constant__ CountArgs a) {
+    extern __shared__ uint32_t s_lane[];                    // kLaneRows x kLaneThreads (residue_classes only)
+    const Col hcol{s_lane + threadIdx.x};
     const uint64_t q_end = a.hdr->small_end;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     uint32_t sK = 0, sH = 0;                                // statistics: WAs by path
@@ -1236,10 +1420,8 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
                     if (g == 0 || g == 128) {
                         lane_uniform(rc, Mk, g != 0, tc, z);
                         sK += Wk;
-                    } else if (d <= 1 && a.residue_classes &&
-                               ((B & 31u) == 0 ||
-                                (((uint32_t(uint64_t(ac.c_par[0])) * B) | (32u * g)) & 127u) == 0)) {
-                        lane_hist1(ac, T0, rc, tc, z);
+                    } else if (d <= 2 && ac.elem_bytes >= 4 && a.residue_classes) {
+                        lane_hist(hcol, ac, T0, T1, uint32_t(nest.P0), B, WR, rc, tc, z);
                         sH += Wk;
                     } else {
                         hmask |= 1u << k;                   // the warp kernel counts access k
@@ -1283,22 +1465,50 @@ __global__ void __launch_bounds__(256) k_lane_problems(const __grid_constant__ C
 // The handed-over accesses of small problems, one warp per queue entry.
 // Entries are taken 32 at a time: lane j loads entry j's problem metadata
 // (independent loads, one latency for the batch), then the warp walks the
-// batch with the metadata broadcast by shuffles and loads only the handed
-// accesses' descriptors.
+// batch with the metadata broadcast by shuffles.  The descriptors of the
+// handed accesses of entry j+1 are copied to shared memory (cp.async, 16 B per
+// request, lane = access) while entry j is counted, so an entry waits for no
+// global load of its own (up to kPrefetch accesses; more read global memory).
+constexpr uint32_t kPrefetch = 8;
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const uint32_t sa = uint32_t(__cvta_generic_to_shared(smem));
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+// lane k (< 31) with bit k of the handed mask and rank r < kPrefetch among the
+// set bits copies descriptor k (64 B) to buf[r]
+__device__ __forceinline__ void prefetch_accesses(sel_access* buf, const sel_access* acc_nest, uint32_t hm, int lane) {
+    if (lane < 31 && ((hm >> lane) & 1u)) {
+        const uint32_t r = uint32_t(__popc(hm & ((1u << lane) - 1u)));
+        if (r < kPrefetch) {
+            const char* src = reinterpret_cast<const char*>(acc_nest + lane);
+            char* dst = reinterpret_cast<char*>(buf + r);
+#pragma unroll
+            for (int c = 0; c < 4; c++) cp_async16(dst + 16 * c, src + 16 * c);
+        }
+    }
+    cp_async_commit();
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_queue(const __grid_constant__ CountArgs a) {
-    const int lane = threadIdx.x & 31;
-    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][128];
-    uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][kHistWords];
+    __shared__ __align__(16) sel_access s_acc[SEL_COUNT_THREADS / 32][2][kPrefetch];
+    uint32_t* hist = a.residue_classes ? s_hist[wid] : nullptr;
     const uint64_t n = a.hdr->queue_len;
-    for (;;) {
-        unsigned long long e0 = 0;
-        if (lane == 0) e0 = atomicAdd(&a.hdr->queue_ctr, 32ull);
-        e0 = __shfl_sync(kFull, e0, 0);
-        if (e0 >= n) break;
+    WarpStats st{0ull, 0ull, 0ull, 0ull};
+    unsigned long long e0 = 0;
+    if (lane == 0) e0 = atomicAdd(&a.hdr->queue_ctr, 32ull);
+    e0 = __shfl_sync(kFull, e0, 0);
+    while (e0 < n) {
         const uint32_t nb = uint32_t(umin64(32, n - e0));
         // lane j: metadata of entry e0 + j
-        uint32_t q_l = 0, hm_l = 0, B_l = 0, WR_l = 0, P_l = 0, T0_l = 0, T1_l = 0, T2_l = 0, ao_l = 0, na_l = 0;
+        uint32_t q_l = 0, hm_l = 0, B_l = 0, WR_l = 0, P_l = 0, T0_l = 0, T1_l = 0, T2_l = 0, ao_l = 0;
         if (uint32_t(lane) < nb) {
             const unsigned long long v = a.queue[e0 + lane];
             q_l = uint32_t(v >> 32);
@@ -1311,8 +1521,12 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
             T1_l = uint32_t(eff_trip(np->trip[1]));
             T2_l = uint32_t(eff_trip(np->trip[2]));
             ao_l = np->access_off;
-            na_l = np->n_access;
         }
+        // the next batch's start, fetched while this one is counted
+        unsigned long long e_next = 0;
+        if (lane == 0) e_next = atomicAdd(&a.hdr->queue_ctr, 32ull);
+        prefetch_accesses(s_acc[wid][0], a.acc + __shfl_sync(kFull, ao_l, 0), __shfl_sync(kFull, hm_l, 0) & 0x7fffffffu,
+                          lane);
         for (uint32_t j = 0; j < nb; j++) {
             const uint32_t q = __shfl_sync(kFull, q_l, j), hmask = __shfl_sync(kFull, hm_l, j);
             const uint32_t B = __shfl_sync(kFull, B_l, j), WR = __shfl_sync(kFull, WR_l, j);
@@ -1320,10 +1534,17 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
             const uint32_t T0 = __shfl_sync(kFull, T0_l, j), T1 = __shfl_sync(kFull, T1_l, j),
                            T2 = __shfl_sync(kFull, T2_l, j);
             const uint32_t aoff = __shfl_sync(kFull, ao_l, j);
+            const uint32_t jn = j + 1 < nb ? j + 1 : j;             // (a dummy copy of j itself at the end)
+            const uint32_t hm_n = __shfl_sync(kFull, hm_l, jn), ao_n = __shfl_sync(kFull, ao_l, jn);
+            prefetch_accesses(s_acc[wid][(j + 1) & 1], a.acc + ao_n, j + 1 < nb ? hm_n & 0x7fffffffu : 0u, lane);
+            cp_async_wait<1>();                                     // entry j's copies have landed
+            __syncwarp();
+            const sel_access* buf = s_acc[wid][j & 1];
             Acc acc{};
-            for (uint32_t mk = hmask & 0x7fffffffu; mk; mk &= mk - 1u) {
+            uint32_t rank = 0;
+            for (uint32_t mk = hmask & 0x7fffffffu; mk; mk &= mk - 1u, rank++) {
                 const uint32_t k = uint32_t(__ffs(mk) - 1);
-                const sel_access* ap = a.acc + aoff + k;
+                const sel_access* ap = rank < kPrefetch ? buf + rank : a.acc + aoff + k;
                 const sel_access ac = *ap;
                 const uint32_t d = ac.depth;
                 const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
@@ -1346,7 +1567,7 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
                 add_part(acc, p);
                 acc.W += Wk;
             }
-            flush(a, q, acc, lane);
+            flush(a, q, acc, lane, st);
             if (hmask >> 31) {                              // accesses 31, 32, ...: the general path
                 uint32_t woff = 0;
                 for (uint32_t k = 0; k < 31; k++) {
@@ -1354,17 +1575,21 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
                     woff += WR * (d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2);
                 }
                 const uint64_t Wq = uint64_t(WR) * a.prob_cnt[uint64_t(q) * kCntStride + 5];
-                count_problem<MODE>(a, q, woff, uint32_t(Wq - woff), lane, hist);
+                count_problem<MODE>(a, q, woff, uint32_t(Wq - woff), lane, hist, st);
             }
+            __syncwarp();                                   // buffer j & 1 is refilled for entry j + 2
         }
-        (void)na_l;
+        cp_async_wait<0>();
+        __syncwarp();
+        e0 = __shfl_sync(kFull, e_next, 0);
     }
+    stats_flush(a, st, lane);
 }
 
 template <int MODE>
 __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_count(const __grid_constant__ CountArgs a) {
     const int lane = threadIdx.x & 31;
-    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][128];
+    __shared__ uint32_t s_hist[SEL_COUNT_THREADS / 32][kHistWords];
     uint32_t* hist = a.residue_classes ? s_hist[threadIdx.x >> 5] : nullptr;
     const uint64_t nq = a.hdr->n_problems;
     if (nq == 0) return;
@@ -1374,6 +1599,7 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
     const uint64_t nwarps = uint64_t(gridDim.x) * (blockDim.x >> 5);
     uint64_t ch = total / (nwarps * 16);
     ch = ch < 256 ? 256 : (ch > kMaxChunk ? kMaxChunk : ch);
+    WarpStats st{0ull, 0ull, 0ull, 0ull};
     for (;;) {
         unsigned long long chunk = 0;
         if (lane == 0) chunk = atomicAdd(&a.hdr->chunk_ctr, 1ull);
@@ -1391,34 +1617,37 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_cou
                 continue;
             }
             const uint32_t take = uint32_t(umin64(Wq - off, len));
-            count_problem<MODE>(a, q, off, take, lane, hist);
+            count_problem<MODE>(a, q, off, take, lane, hist, st);
             len -= take;
             off = 0;
             q++;
         }
     }
+    stats_flush(a, st, lane);
 }
 
 // persistent grid: #SMs x resident blocks of kernel k
 template <typename K>
-static int persistent_grid(K k, int threads) {
+static int persistent_grid(K k, int threads, size_t smem = 0) {
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, threads, 0);
+    if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, threads, smem);
     return sms * (per > 0 ? per : 1);
 }
 
 template <int MODE>
 static void launch_mode(const CountArgs& a, cudaStream_t s) {
     static int g_count = 0, g_queue = 0, g_lane = 0;
+    const size_t lane_smem = a.residue_classes ? size_t(kLaneRows) * kLaneThreads * sizeof(uint32_t) : 0;
     if (g_count == 0) {
         g_count = persistent_grid(k_count<MODE>, SEL_COUNT_THREADS);
         g_queue = persistent_grid(k_queue<MODE>, SEL_COUNT_THREADS);
-        g_lane = persistent_grid(k_lane_problems<MODE>, 256);
+        g_lane = persistent_grid(k_lane_problems<MODE>, kLaneThreads, size_t(kLaneRows) * kLaneThreads * sizeof(uint32_t));
     }
     if (MODE != 0) {
-        k_lane_problems<MODE><<<g_lane, 256, 0, s>>>(a);
+        k_lane_problems<MODE><<<g_lane, kLaneThreads, lane_smem, s>>>(a);
         k_queue<MODE><<<g_queue, SEL_COUNT_THREADS, 0, s>>>(a);
         note_launch(2);
     }

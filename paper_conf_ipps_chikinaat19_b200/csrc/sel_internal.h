@@ -22,6 +22,8 @@ struct WsPtrs {
     uint8_t* prob_status;
     uint8_t* cand_status;
     unsigned long long* queue;       // (problem << 32 | first WA) handed from the lane to the warp kernel
+    void* prob_md;                   // per problem: ProbModel (sel_model.cu)
+    uint32_t* cls;                   // [kClsMax] class index per launch, [kClsMax..) B class per index
     unsigned long long* scan_tmp;
 };
 

@@ -128,13 +128,64 @@ static cudaError_t scan_u64(unsigned long long* x, uint64_t n_max, const unsigne
 }
 
 // ------------------------------------------------------------------ plan
-// V1-V2 per candidate; dedup: insert the candidate's B class into its nest's
-// slot table (one CAS per distinct key per warp).
+// Direct problem ids (launch tables of <= kClsMax entries whose nests x
+// classes fit the workspace): the distinct B classes of the launch table,
+// sorted, give every launch a class index, and problem = nest * n_cls +
+// class index -- deterministic, no slot table, no second pass over the
+// candidates.  Problems no candidate refers to keep prob_nest = kNoProblem
+// and are skipped.  One block; O(n_launches^2) comparisons.
+__global__ void __launch_bounds__(1024) k_classes(sel_tables t, uint64_t n, uint64_t n_nests, int dedup,
+                                                  WsHeader* hdr, uint32_t* cls) {
+    __shared__ uint32_t s_bc[kClsMax];
+    __shared__ uint8_t s_first[kClsMax];
+    __shared__ uint32_t s_ncls;
+    const uint64_t nl = t.n_launches;
+    if (!dedup || nl == 0 || nl > kClsMax) {
+        if (threadIdx.x == 0) {
+            hdr->direct = 0;
+            hdr->n_nests_scan = n_nests;
+        }
+        return;
+    }
+    if (threadIdx.x == 0) s_ncls = 0;
+    for (uint32_t i = threadIdx.x; i < nl; i += blockDim.x) s_bc[i] = b_class(t.launches[i].block);
+    __syncthreads();
+    uint32_t nf = 0;
+    for (uint32_t i = threadIdx.x; i < nl; i += blockDim.x) {
+        uint8_t first = 1;
+        for (uint32_t j = 0; j < i; j++)
+            if (s_bc[j] == s_bc[i]) { first = 0; break; }
+        s_first[i] = first;
+        nf += first;
+    }
+    atomicAdd(&s_ncls, nf);
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < nl; i += blockDim.x) {
+        uint32_t rank = 0;
+        for (uint32_t j = 0; j < nl; j++) rank += (s_first[j] && s_bc[j] < s_bc[i]) ? 1u : 0u;
+        cls[i] = rank;
+        if (s_first[i]) cls[kClsMax + rank] = s_bc[i];
+    }
+    if (threadIdx.x == 0) {
+        const uint64_t ncls = s_ncls;
+        const bool direct = n_nests * ncls <= n;
+        hdr->direct = direct ? 1u : 0u;
+        hdr->n_cls = uint32_t(ncls);
+        hdr->n_nests_scan = direct ? 0ull : n_nests;
+    }
+}
+
+// V1-V2 per candidate; dedup: the candidate's problem id directly (direct
+// mode), or insert its B class into its nest's slot table (one CAS per
+// distinct key per warp).
 __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict__ cands, uint64_t n,
                                                 sel_tables t, int n_sets, uint32_t* slots,
                                                 uint8_t* cand_status, int dedup, uint32_t* prob_nest,
-                                                uint32_t* prob_B, uint32_t* cand_pid) {
+                                                uint32_t* prob_B, uint32_t* cand_pid, const WsHeader* hdr,
+                                                const uint32_t* cls) {
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    const bool direct = dedup && hdr->direct;
+    const uint32_t ncls = hdr->n_cls;
     for (uint64_t base = uint64_t(blockIdx.x) * blockDim.x; base < n; base += stride) {
         const uint64_t c = base + threadIdx.x;
         const bool in = c < n;
@@ -143,6 +194,18 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
         const sel_candidate cd = cands[c];
         const uint8_t st = validate_candidate(cd, t, n_sets);
         cand_status[c] = st;
+        if (direct) {
+            const uint32_t ci = st ? 0u : cls[cd.launch_id];
+            const uint32_t pid = st ? kNoProblem : cd.nest_id * ncls + ci;
+            cand_pid[c] = pid;
+            // identical values from every sharer: one write per distinct problem of the warp
+            const unsigned peers = __match_any_sync(inmask, pid);
+            if (!st && int(threadIdx.x & 31) == __ffs(peers) - 1) {
+                prob_nest[pid] = cd.nest_id;
+                prob_B[pid] = cls[kClsMax + ci];
+            }
+            continue;
+        }
         if (!dedup) {
             cand_pid[c] = uint32_t(c);
             prob_nest[c] = st ? kNoProblem : cd.nest_id;
@@ -168,9 +231,9 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
 
 // sort each nest's B classes (deterministic ids) and count them
 __global__ void __launch_bounds__(256) k_rank_slots(uint32_t* slots, uint64_t n_nests,
-                                                    unsigned long long* nest_cnt) {
+                                                    unsigned long long* nest_cnt, const WsHeader* hdr) {
     const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (i >= n_nests) return;
+    if (i >= n_nests || hdr->direct) return;
     uint32_t v[kSlots];
     int m = 0;
     for (int j = 0; j < kSlots; j++) {
@@ -187,13 +250,10 @@ __global__ void __launch_bounds__(256) k_rank_slots(uint32_t* slots, uint64_t n_
     nest_cnt[i] = (unsigned long long)m;
 }
 
-__global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict__ cands, uint64_t n,
-                                                sel_tables t, const uint32_t* slots,
-                                                const unsigned long long* nest_base, uint64_t n_nests,
-                                                const uint8_t* cand_status, uint32_t* cand_pid,
-                                                uint32_t* prob_nest, uint32_t* prob_B, WsHeader* hdr) {
-    const uint64_t c = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (c >= n) return;
+__device__ __forceinline__ void assign_one(const sel_candidate* __restrict__ cands, uint64_t c, const sel_tables& t,
+                                           const uint32_t* slots, const unsigned long long* nest_base,
+                                           uint64_t n_nests, const uint8_t* cand_status, uint32_t* cand_pid,
+                                           uint32_t* prob_nest, uint32_t* prob_B, WsHeader* hdr) {
     if (cand_status[c]) { cand_pid[c] = kNoProblem; return; }
     const sel_candidate cd = cands[c];
     const uint32_t bc = b_class(t.launches[cd.launch_id].block);
@@ -212,40 +272,59 @@ __global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict_
     }
 }
 
+__global__ void __launch_bounds__(256) k_assign(const sel_candidate* __restrict__ cands, uint64_t n,
+                                                sel_tables t, const uint32_t* slots,
+                                                const unsigned long long* nest_base, uint64_t n_nests,
+                                                const uint8_t* cand_status, uint32_t* cand_pid,
+                                                uint32_t* prob_nest, uint32_t* prob_B, WsHeader* hdr) {
+    if (hdr->direct) return;
+    for (uint64_t c = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; c < n; c += uint64_t(gridDim.x) * blockDim.x)
+        assign_one(cands, c, t, slots, nest_base, n_nests, cand_status, cand_pid, prob_nest, prob_B, hdr);
+}
 __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_base, uint64_t n_nests,
                                 uint64_t n, int dedup, uint32_t part, uint32_t n_parts) {
-    unsigned long long np = dedup ? nest_base[n_nests] + hdr->n_overflow : n;
+    const bool direct = dedup && hdr->direct;
+    unsigned long long np = !dedup ? n : direct ? n_nests * hdr->n_cls : nest_base[n_nests] + hdr->n_overflow;
     hdr->n_problems = np;
     hdr->part = part;
     hdr->n_parts = n_parts;
     hdr->chunk_ctr = 0;
     hdr->stats.n_candidates = n;
-    hdr->stats.n_problems = np;
+    hdr->stats.n_problems = direct ? 0ull : np;        // direct mode: k_problem_w counts the used ids
 }
 
 // closed-form W = WR * M_it per problem (+ nest validation V3-V6)
-__global__ void __launch_bounds__(256) k_problem_w(sel_tables t, const WsHeader* hdr, const uint32_t* prob_nest,
+__global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
                                                    unsigned long long* prob_cnt, int lane_ok) {
     const uint64_t nq = hdr->n_problems;
-    const uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (q >= nq) return;
-    for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
-    const uint32_t nid = prob_nest[q];
-    if (nid == kNoProblem) { prob_W[q] = 0; prob_WR[q] = 0; prob_status[q] = SEL_EINVAL; return; }
-    const sel_nest nest = t.nests[nid];
-    uint64_t M_it = 0;
-    const uint8_t st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
-    prob_status[q] = st;
-    if (st) { prob_W[q] = 0; prob_WR[q] = 0; return; }
-    const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
-    prob_WR[q] = WR;
-    prob_cnt[q * kCntStride + 5] = M_it;
-    // small problems are counted one per lane (k_lane_problems), outside the prefix
-    const uint64_t W = WR * M_it;
-    const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
-    prob_W[q] = small ? 0ull : W;
+    const bool direct = hdr->direct;
+    uint32_t used = 0;
+    // grid-stride: the grid is sized for the candidates, the problems (known on
+    // the device only) are usually an order of magnitude fewer
+    for (uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; q < nq; q += uint64_t(gridDim.x) * blockDim.x) {
+        for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
+        const uint32_t nid = prob_nest[q];
+        if (nid == kNoProblem) { prob_W[q] = 0; prob_WR[q] = 0; prob_status[q] = SEL_EINVAL; continue; }
+        used++;
+        const sel_nest nest = t.nests[nid];
+        uint64_t M_it = 0;
+        const uint8_t st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
+        prob_status[q] = st;
+        if (st) { prob_W[q] = 0; prob_WR[q] = 0; continue; }
+        const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
+        prob_WR[q] = WR;
+        prob_cnt[q * kCntStride + 5] = M_it;
+        // small problems are counted one per lane (k_lane_problems), outside the prefix
+        const uint64_t W = WR * M_it;
+        const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
+        prob_W[q] = small ? 0ull : W;
+    }
+    if (direct) {
+        used = __reduce_add_sync(kFull, used);
+        if ((threadIdx.x & 31) == 0 && used) atomicAdd((unsigned long long*)&hdr->stats.n_problems, (unsigned long long)used);
+    }
 }
 
 // slice [total*part/n_parts, total*(part+1)/n_parts) of the problem work space
@@ -273,24 +352,28 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
     if (dedup && n_nests) {
         e = cudaMemsetAsync(w.slots, 0, n_nests * kSlots * sizeof(uint32_t), s);
         if (e != cudaSuccess) return e;
+        // direct mode: problem ids no candidate refers to stay kNoProblem
+        const uint64_t ids = n_nests * (t.n_launches < kClsMax ? t.n_launches : kClsMax);
+        e = cudaMemsetAsync(w.prob_nest, 0xff, (ids < n ? ids : n) * sizeof(uint32_t), s);
+        if (e != cudaSuccess) return e;
     }
+    k_classes<<<1, 1024, 0, s>>>(t, n, n_nests, dedup ? 1 : 0, w.hdr, w.cls);
     const unsigned gb = unsigned((n + 255) / 256 < 148u * 64 ? (n + 255) / 256 : 148u * 64);
     k_insert<<<gb, 256, 0, s>>>(cands, n, t, n_sets, w.slots, w.cand_status, dedup ? 1 : 0, w.prob_nest,
-                                w.prob_B, w.cand_pid);
-    note_launch();
+                                w.prob_B, w.cand_pid, w.hdr, w.cls);
+    note_launch(2);
     if (dedup) {
         if (n_nests) {
-            k_rank_slots<<<unsigned((n_nests + 255) / 256), 256, 0, s>>>(w.slots, n_nests, w.nest_base);
+            k_rank_slots<<<unsigned((n_nests + 255) / 256), 256, 0, s>>>(w.slots, n_nests, w.nest_base, w.hdr);
             note_launch();
         }
-        if ((e = scan_u64(w.nest_base, n_nests, nullptr, w.scan_tmp, s)) != cudaSuccess) return e;
-        k_assign<<<unsigned((n + 255) / 256), 256, 0, s>>>(cands, n, t, w.slots, w.nest_base, n_nests,
-                                                           w.cand_status, w.cand_pid, w.prob_nest, w.prob_B,
-                                                           w.hdr);
+        if ((e = scan_u64(w.nest_base, n_nests, &w.hdr->n_nests_scan, w.scan_tmp, s)) != cudaSuccess) return e;
+        k_assign<<<gb, 256, 0, s>>>(cands, n, t, w.slots, w.nest_base, n_nests, w.cand_status, w.cand_pid,
+                                    w.prob_nest, w.prob_B, w.hdr);
         note_launch();
     }
     k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0, part, n_parts);
-    k_problem_w<<<unsigned((n + 255) / 256), 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
+    k_problem_w<<<gb, 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
                                                           w.prob_status, w.prob_cnt,
                                                           (flags & (SEL_F_MATCH_ANY | SEL_F_EXPAND_ALL |
                                                                     SEL_F_WARP_PROBLEMS)) ? 0 : 1);

@@ -1,0 +1,10 @@
+# one GPU call: build, GPU tests, bench, launch list, ncu --set full of the three counting kernels (c5 full size)
+mkdir -p gpurun_out
+python __graft_entry__.py
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/tests.log 2>&1
+timeout 600 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.json 2> gpurun_out/bench.err
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
+    python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --no-next > gpurun_out/ncu_launch_bench.json 2>&1
+timeout 1800 ncu --set full --clock-control none --import-source on -k 'regex:k_count|k_queue|k_lane_problems' -s 9 -c 3 -o gpurun_out/prof_count_full \
+    python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --no-next > gpurun_out/ncu_full.log 2>&1
+tail -3 gpurun_out/tests.log; cat gpurun_out/bench.json; tail -3 gpurun_out/bench.err; tail -2 gpurun_out/ncu_full.log

@@ -55,7 +55,6 @@ constexpr uint32_t kOpsArithWA = 12;     // arithmetic lanes, per WA: residue 2,
 constexpr uint32_t kOpsClass = 6;        // uniform flags, per (access, lane-count class): lines, class, 4 sums
 constexpr uint32_t kOpsHistEntry = 6;    // residue histogram of one loop, per entry: residue 3, count 3
 constexpr uint32_t kOpsConvTerm = 5;     // histogram convolution, per (iteration, residue): index 4, MAC 1
-constexpr uint32_t kOpsEvalTerm = 12;    // residue-class evaluation, per (class, residue): as an arithmetic WA
 constexpr uint32_t kOpsPrefixEntry = 3;  // prefix sums of a residue histogram, per entry
 constexpr uint32_t kOpsEvalClass = 24;   // one residue class from the prefix sums: 2 cyclic range sums + sums
 // per-warp shared words of a residue histogram: h / its exclusive prefix pf[0..R]
@@ -1331,12 +1330,18 @@ __device__ __forceinline__ void lane_add(LaneSums& z, const ClassSums& c, uint32
     z.U += (w - c.cc) + c.uf;
 }
 
-// one access (depth <= 2, E >= 4, 0 < |c_par| < 128) of a small problem
-__device__ __forceinline__ void lane_hist(Col h, const sel_access& a, uint32_t T0, uint32_t T1, uint32_t P, uint32_t B,
-                                          uint32_t WR, const RepClasses& rc, uint32_t tmin, LaneSums& z) {
+// one access (depth <= 2, E >= 4, 0 < |c_par| < 128): its residue histogram
+// and prefix sums in the thread's column (shared by every block size class
+// of the nest), then the warp-rep classes of one problem (B, WR, rc)
+__device__ __forceinline__ void lane_hist_prepare(Col h, const sel_access& a, uint32_t T0, uint32_t T1,
+                                                  unsigned long long& ops) {
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
-    lane_hist_build(h, R, sh, a, T0, T1, z.ops);
-    lane_hist_prefix(h, R, z.ops);
+    lane_hist_build(h, R, sh, a, T0, T1, ops);
+    lane_hist_prefix(h, R, ops);
+}
+__device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint32_t P, uint32_t B, uint32_t WR,
+                                               const RepClasses& rc, uint32_t tmin, LaneSums& z) {
+    const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
     const Col p32{h.p + kLaneP32 * kLaneThreads};
     const uint32_t Ht = h[R];                               // = Mk
     const int64_t c0 = a.c_par[0];
@@ -1378,83 +1383,184 @@ __device__ __forceinline__ void lane_hist(Col h, const sel_access& a, uint32_t T
 }
 
 // Small problems (k_problem_w: 1-D, W <= kSmallMaxW, WR <= kSmallMaxWR), one
-// per thread, grid-stride over this call's problem range.  A thread hands the
-// rest of its problem to the warp kernel (k_queue) at the first access that
-// needs a warp: entry = problem << 32 | WA offset of that access.
+// UNIT per thread: a nest with all of its block size classes in direct mode
+// (problems u * n_cls + c; the classes share the nest's residue histograms),
+// one problem otherwise.  A block takes a tile of kLaneTile units and sorts
+// them by a shape key (accesses, loop depth, collapse) in shared memory, so a
+// warp's lanes run nests of one shape side by side instead of 32 different
+// loop structures.  A thread hands the accesses it cannot count to the warp
+// kernel (k_queue): entry = problem << 32 | mask of handed accesses.
+#ifndef SEL_LANE_MIN_BLOCKS
+#define SEL_LANE_MIN_BLOCKS 2
+#endif
+constexpr uint32_t kLaneGrp = 4;        // problems of a unit counted together
+constexpr uint32_t kLaneTile = 2048;    // units sorted per block tile
+constexpr uint32_t kLaneKeys = 256;
+constexpr size_t kLaneSmem = (size_t(kLaneRows) * kLaneThreads + kLaneTile + kLaneKeys) * sizeof(uint32_t);
+
+__device__ __forceinline__ uint32_t lane_unit_key(const CountArgs& a, uint64_t u, bool direct) {
+    const uint32_t nid = direct ? uint32_t(u) : a.prob_nest[u];
+    if (nid == kNoProblem) return 0u;
+    const sel_nest* np = a.nests + nid;
+    const uint32_t na = np->n_access < 31u ? np->n_access : 31u;
+    return (na << 3) | (uint32_t(np->depth & 3u) << 1) | (np->par_dims == 2 ? 1u : 0u);
+}
+
 template <int MODE>
-__global__ void __launch_bounds__(kLaneThreads) k_lane_problems(const __grid_constant__ CountArgs a) {
-    extern __shared__ uint32_t s_lane[];                    // kLaneRows x kLaneThreads (residue_classes only)
+__global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_problems(const __grid_constant__ CountArgs a) {
+    extern __shared__ uint32_t s_lane[];                    // hist columns | tile order | key counts
+    uint32_t* s_order = s_lane + kLaneRows * kLaneThreads;
+    uint32_t* s_cnt = s_order + kLaneTile;
     const Col hcol{s_lane + threadIdx.x};
-    const uint64_t q_end = a.hdr->small_end;
-    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    const int lane = threadIdx.x & 31;
+    const bool direct = a.hdr->direct != 0;
+    const uint32_t ncls = direct ? a.hdr->n_cls : 1u;
+    const uint64_t qb = a.hdr->small_begin, qe = a.hdr->small_end;
+    const uint64_t ub = qb / ncls, ue = (qe + ncls - 1) / ncls;
     uint32_t sK = 0, sH = 0;                                // statistics: WAs by path
     unsigned long long sW = 0, sOps = 0;
-    for (uint64_t qb = a.hdr->small_begin + uint64_t(blockIdx.x) * blockDim.x; qb < q_end; qb += stride) {
-        const uint64_t q = qb + threadIdx.x;
-        uint32_t hmask = 0;                                 // accesses handed to the warp kernel
-        if (q < q_end && a.prefix[q + 1] == a.prefix[q]) {
-            const uint64_t WR64 = a.prob_WR[q];
-            const uint64_t Wq = WR64 * a.prob_cnt[q * kCntStride + 5];
-            if (Wq) {                                       // small (valid, outside the prefix)
-                sW += Wq;
-                const sel_nest nest = a.nests[a.prob_nest[q]];
-                const uint32_t B = a.prob_B[q];
-                const uint32_t WR = uint32_t(WR64);
-                const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
-                               T2 = uint32_t(eff_trip(nest.trip[2]));
-                const RepClasses rc = rep_classes(nest.P0, B);
-                LaneSums z{0u, 0u, 0u, 0u, 0u, 0ull};
-                const sel_access* ap = a.acc + nest.access_off;
-                for (uint32_t k = 0; k < nest.n_access; k++, ap++) {
-                    if (k == 31) {                          // accesses 31, 32, ...: all to the warp kernel
-                        hmask |= 1u << 31;
-                        break;
+    for (uint64_t t0 = ub + uint64_t(blockIdx.x) * kLaneTile; t0 < ue; t0 += uint64_t(gridDim.x) * kLaneTile) {
+        const uint32_t nt = uint32_t(umin64(kLaneTile, ue - t0));
+        // ---- sort the tile's units by shape key (counting sort in shared memory)
+        for (uint32_t i = threadIdx.x; i < kLaneKeys; i += blockDim.x) s_cnt[i] = 0u;
+        __syncthreads();
+        uint32_t key[kLaneTile / kLaneThreads];
+#pragma unroll
+        for (uint32_t r = 0; r < kLaneTile / kLaneThreads; r++) {
+            const uint32_t i = r * kLaneThreads + threadIdx.x;
+            key[r] = i < nt ? lane_unit_key(a, t0 + i, direct) : 0u;
+            if (i < nt) atomicAdd(&s_cnt[key[r]], 1u);
+        }
+        __syncthreads();
+        if (threadIdx.x < 32) {                             // exclusive scan of the 256 key counts
+            uint32_t v[kLaneKeys / 32], sum = 0;
+#pragma unroll
+            for (uint32_t j = 0; j < kLaneKeys / 32; j++) { v[j] = s_cnt[threadIdx.x * (kLaneKeys / 32) + j]; sum += v[j]; }
+            uint32_t x = sum;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, x, o);
+                if (lane >= o) x += y;
+            }
+            uint32_t run = x - sum;
+#pragma unroll
+            for (uint32_t j = 0; j < kLaneKeys / 32; j++) { s_cnt[threadIdx.x * (kLaneKeys / 32) + j] = run; run += v[j]; }
+        }
+        __syncthreads();
+#pragma unroll
+        for (uint32_t r = 0; r < kLaneTile / kLaneThreads; r++) {
+            const uint32_t i = r * kLaneThreads + threadIdx.x;
+            if (i < nt) s_order[atomicAdd(&s_cnt[key[r]], 1u)] = i;
+        }
+        __syncthreads();
+        // ---- count: round r, thread t takes the unit at sorted position r * threads + t
+        for (uint32_t r = 0; r * kLaneThreads < nt; r++) {
+            const uint32_t i = r * kLaneThreads + threadIdx.x;
+            const bool has = i < nt;
+            const uint64_t u = has ? t0 + s_order[i] : 0ull;
+            for (uint32_t g0 = 0; g0 < ncls; g0 += kLaneGrp) {
+                // problems q = u * ncls + g0 + c of this group that are small and in this call's range
+                uint32_t B[kLaneGrp], WR[kLaneGrp], hm[kLaneGrp];
+                RepClasses rc[kLaneGrp];
+                LaneSums z[kLaneGrp];
+                uint32_t vmask = 0;
+                sel_nest nest{};
+                if (has) {
+#pragma unroll
+                    for (uint32_t c = 0; c < kLaneGrp; c++) {
+                        hm[c] = 0u;
+                        z[c] = LaneSums{0u, 0u, 0u, 0u, 0u, 0ull};
+                        B[c] = 0u;
+                        WR[c] = 0u;
+                        rc[c] = RepClasses{0ull, 0ull, 0u, 0u};
+                        const uint64_t q = u * ncls + g0 + c;
+                        if (g0 + c < ncls && q >= qb && q < qe && a.prefix[q + 1] == a.prefix[q]) {
+                            const uint64_t WR64 = a.prob_WR[q];
+                            if (WR64 * a.prob_cnt[q * kCntStride + 5]) {      // small, valid, W > 0
+                                vmask |= 1u << c;
+                                WR[c] = uint32_t(WR64);
+                                B[c] = a.prob_B[q];
+                            }
+                        }
                     }
-                    const sel_access ac = *ap;
-                    const uint32_t d = ac.depth;
-                    const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
-                    const uint32_t Wk = WR * Mk;
-                    if (Wk == 0) continue;
-                    const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
-                    const uint32_t g = uint32_t(umin64(uabs(ac.c_par[0]), 128));
-                    if (g == 0 || g == 128) {
-                        lane_uniform(rc, Mk, g != 0, tc, z);
-                        sK += Wk;
-                    } else if (d <= 2 && ac.elem_bytes >= 4 && a.residue_classes) {
-                        lane_hist(hcol, ac, T0, T1, uint32_t(nest.P0), B, WR, rc, tc, z);
-                        sH += Wk;
-                    } else {
-                        hmask |= 1u << k;                   // the warp kernel counts access k
-                        continue;
-                    }
-                    z.W += Wk;
                 }
-                sOps += z.ops;
-                if (z.W) {
-                    unsigned long long* pc = a.prob_cnt + q * kCntStride;
-                    atomicAdd(pc + 0, (unsigned long long)z.W);
-                    atomicAdd(pc + 1, (unsigned long long)z.L);
-                    atomicAdd(pc + 2, (unsigned long long)z.S);
-                    atomicAdd(pc + 3, (unsigned long long)z.C);
-                    atomicAdd(pc + 4, (unsigned long long)z.U);
+                if (vmask) {
+                    nest = a.nests[direct ? uint32_t(u) : a.prob_nest[u]];
+#pragma unroll
+                    for (uint32_t c = 0; c < kLaneGrp; c++)
+                        if ((vmask >> c) & 1u) rc[c] = rep_classes(nest.P0, B[c]);
+                    const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
+                                   T2 = uint32_t(eff_trip(nest.trip[2]));
+                    const sel_access* ap = a.acc + nest.access_off;
+                    for (uint32_t k = 0; k < nest.n_access; k++, ap++) {
+                        if (k == 31) {                      // accesses 31, 32, ...: all to the warp kernel
+#pragma unroll
+                            for (uint32_t c = 0; c < kLaneGrp; c++) hm[c] |= ((vmask >> c) & 1u) << 31;
+                            break;
+                        }
+                        const sel_access ac = *ap;
+                        const uint32_t d = ac.depth;
+                        const uint32_t Mk = d == 0 ? 1u : d == 1 ? T0 : d == 2 ? T0 * T1 : T0 * T1 * T2;
+                        if (Mk == 0) continue;
+                        const uint32_t tc = ac.elem_bytes <= 4 ? 1u : ac.elem_bytes == 8 ? 2u : 4u;   // R11
+                        const uint32_t g = uint32_t(umin64(uabs(ac.c_par[0]), 128));
+                        if (g == 0 || g == 128) {
+#pragma unroll
+                            for (uint32_t c = 0; c < kLaneGrp; c++)
+                                if ((vmask >> c) & 1u) {
+                                    lane_uniform(rc[c], Mk, g != 0, tc, z[c]);
+                                    sK += WR[c] * Mk;
+                                    z[c].W += WR[c] * Mk;
+                                }
+                        } else if (d <= 2 && ac.elem_bytes >= 4 && a.residue_classes) {
+                            lane_hist_prepare(hcol, ac, T0, T1, z[0].ops);
+#pragma unroll
+                            for (uint32_t c = 0; c < kLaneGrp; c++)
+                                if ((vmask >> c) & 1u) {
+                                    lane_hist_eval(hcol, ac, uint32_t(nest.P0), B[c], WR[c], rc[c], tc, z[c]);
+                                    sH += WR[c] * Mk;
+                                    z[c].W += WR[c] * Mk;
+                                }
+                        } else {
+#pragma unroll
+                            for (uint32_t c = 0; c < kLaneGrp; c++) hm[c] |= ((vmask >> c) & 1u) << k;   // to k_queue
+                        }
+                    }
+#pragma unroll
+                    for (uint32_t c = 0; c < kLaneGrp; c++) {
+                        if (!((vmask >> c) & 1u)) continue;
+                        const uint64_t q = u * ncls + g0 + c;
+                        sW += uint64_t(WR[c]) * a.prob_cnt[q * kCntStride + 5];
+                        sOps += z[c].ops;
+                        if (z[c].W) {
+                            unsigned long long* pc = a.prob_cnt + q * kCntStride;
+                            atomicAdd(pc + 0, (unsigned long long)z[c].W);
+                            atomicAdd(pc + 1, (unsigned long long)z[c].L);
+                            atomicAdd(pc + 2, (unsigned long long)z[c].S);
+                            atomicAdd(pc + 3, (unsigned long long)z[c].C);
+                            atomicAdd(pc + 4, (unsigned long long)z[c].U);
+                        }
+                    }
+                }
+                // warp-aggregated append of the handed problems to the queue (converged)
+#pragma unroll
+                for (uint32_t c = 0; c < kLaneGrp; c++) {
+                    const bool enq = ((vmask >> c) & 1u) && hm[c] != 0u;
+                    const unsigned m = __ballot_sync(kFull, enq);
+                    if (m) {
+                        unsigned long long base = 0;
+                        if (lane == __ffs(m) - 1) base = atomicAdd(&a.hdr->queue_len, (unsigned long long)__popc(m));
+                        base = __shfl_sync(kFull, base, __ffs(m) - 1);
+                        if (enq) a.queue[base + __popc(m & lanemask_lt())] = ((u * ncls + g0 + c) << 32) | hm[c];
+                    }
                 }
             }
         }
-        // warp-aggregated append to the queue
-        const bool enq = hmask != 0;
-        const unsigned m = __ballot_sync(kFull, enq);
-        if (m) {
-            unsigned long long base = 0;
-            const int lane = threadIdx.x & 31;
-            if (lane == __ffs(m) - 1) base = atomicAdd(&a.hdr->queue_len, (unsigned long long)__popc(m));
-            base = __shfl_sync(kFull, base, __ffs(m) - 1);
-            if (enq) a.queue[base + __popc(m & lanemask_lt())] = (q << 32) | hmask;
-        }
+        __syncthreads();                                    // s_order / s_cnt are rewritten by the next tile
     }
     const uint32_t K = __reduce_add_sync(kFull, sK), H = __reduce_add_sync(kFull, sH);
     unsigned long long Wt = sW;
     for (int o = 16; o; o >>= 1) Wt += __shfl_xor_sync(kFull, Wt, o);
-    const int lane = threadIdx.x & 31;
     if (K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)K);
     if (H && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)H);
     if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_analysed, Wt);
@@ -1640,11 +1746,11 @@ static int persistent_grid(K k, int threads, size_t smem = 0) {
 template <int MODE>
 static void launch_mode(const CountArgs& a, cudaStream_t s) {
     static int g_count = 0, g_queue = 0, g_lane = 0;
-    const size_t lane_smem = a.residue_classes ? size_t(kLaneRows) * kLaneThreads * sizeof(uint32_t) : 0;
+    const size_t lane_smem = kLaneSmem;
     if (g_count == 0) {
         g_count = persistent_grid(k_count<MODE>, SEL_COUNT_THREADS);
         g_queue = persistent_grid(k_queue<MODE>, SEL_COUNT_THREADS);
-        g_lane = persistent_grid(k_lane_problems<MODE>, kLaneThreads, size_t(kLaneRows) * kLaneThreads * sizeof(uint32_t));
+        g_lane = persistent_grid(k_lane_problems<MODE>, kLaneThreads, kLaneSmem);
     }
     if (MODE != 0) {
         k_lane_problems<MODE><<<g_lane, kLaneThreads, lane_smem, s>>>(a);

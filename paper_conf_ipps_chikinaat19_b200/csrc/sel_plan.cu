@@ -294,36 +294,68 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 }
 
 // closed-form W = WR * M_it per problem (+ nest validation V3-V6)
+__device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
+                                              const uint32_t* prob_B, unsigned long long* prob_W,
+                                              unsigned long long* prob_WR, uint8_t* prob_status,
+                                              unsigned long long* prob_cnt, int lane_ok) {
+    for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
+    prob_status[q] = st;
+    if (st) { prob_W[q] = 0; prob_WR[q] = 0; prob_cnt[q * kCntStride + 5] = 0; return; }
+    const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
+    prob_WR[q] = WR;
+    prob_cnt[q * kCntStride + 5] = M_it;
+    // small problems are counted one per lane (k_lane_problems), outside the prefix
+    const uint64_t W = WR * M_it;
+    const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
+    prob_W[q] = small ? 0ull : W;
+}
+
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
                                                    unsigned long long* prob_cnt, int lane_ok) {
     const uint64_t nq = hdr->n_problems;
-    const bool direct = hdr->direct;
-    uint32_t used = 0;
-    // grid-stride: the grid is sized for the candidates, the problems (known on
-    // the device only) are usually an order of magnitude fewer
-    for (uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; q < nq; q += uint64_t(gridDim.x) * blockDim.x) {
-        for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
-        const uint32_t nid = prob_nest[q];
-        if (nid == kNoProblem) { prob_W[q] = 0; prob_WR[q] = 0; prob_status[q] = SEL_EINVAL; continue; }
-        used++;
-        const sel_nest nest = t.nests[nid];
-        uint64_t M_it = 0;
-        const uint8_t st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
-        prob_status[q] = st;
-        if (st) { prob_W[q] = 0; prob_WR[q] = 0; continue; }
-        const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
-        prob_WR[q] = WR;
-        prob_cnt[q * kCntStride + 5] = M_it;
-        // small problems are counted one per lane (k_lane_problems), outside the prefix
-        const uint64_t W = WR * M_it;
-        const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
-        prob_W[q] = small ? 0ull : W;
-    }
-    if (direct) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    if (hdr->direct) {
+        // direct ids: the problems of nest i are i * n_cls + [0, n_cls) -- one thread
+        // per nest validates it once for all of them
+        const uint32_t ncls = hdr->n_cls;
+        const uint64_t nn = ncls ? nq / ncls : 0;
+        uint32_t used = 0;
+        for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < nn; i += stride) {
+            uint32_t um = 0;
+            for (uint32_t c = 0; c < ncls; c++) um |= (prob_nest[i * ncls + c] != kNoProblem ? 1u : 0u) << (c & 31u);
+            sel_nest nest{};
+            uint64_t M_it = 0;
+            uint8_t st = SEL_EINVAL;
+            if (um) {
+                nest = t.nests[i];
+                st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
+            }
+            for (uint32_t c = 0; c < ncls; c++) {
+                const uint64_t q = i * ncls + c;
+                const bool u = c < 32 ? ((um >> c) & 1u) : prob_nest[q] != kNoProblem;
+                used += u ? 1u : 0u;
+                problem_w_one(q, nest, u ? st : uint8_t(SEL_EINVAL), M_it, prob_B, prob_W, prob_WR, prob_status,
+                              prob_cnt, lane_ok);
+            }
+        }
         used = __reduce_add_sync(kFull, used);
         if ((threadIdx.x & 31) == 0 && used) atomicAdd((unsigned long long*)&hdr->stats.n_problems, (unsigned long long)used);
+        return;
+    }
+    // grid-stride: the grid is sized for the candidates, the problems (known on
+    // the device only) are usually an order of magnitude fewer
+    for (uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; q < nq; q += stride) {
+        const uint32_t nid = prob_nest[q];
+        sel_nest nest{};
+        uint64_t M_it = 0;
+        uint8_t st = SEL_EINVAL;
+        if (nid != kNoProblem) {
+            nest = t.nests[nid];
+            st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
+        }
+        problem_w_one(q, nest, st, M_it, prob_B, prob_W, prob_WR, prob_status, prob_cnt, lane_ok);
     }
 }
 

@@ -114,45 +114,70 @@ __device__ __forceinline__ uint8_t validate_candidate(const sel_candidate& c, co
     return SEL_OK;
 }
 
-// Nest-level checks V3-V6; on success *M_it = sum_k prod_{j<depth_k} T_j.
-__device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc_all, uint64_t n_acc_total,
-                                        uint64_t* M_it_out) {
+// Nest-level checks V3-V6, split so that the accesses can be checked by
+// different threads: nest_precheck (structure, P range), access_check (one
+// access: element size, depth, divisibility -> kAccInval; address bound ->
+// kAccRange; its Mk), nest_status (combines them in validate_nest's order:
+// a structural error of any access wins over a range error).
+constexpr uint32_t kAccInval = 1u, kAccRange = 2u;
+__device__ __forceinline__ uint8_t nest_precheck(const sel_nest& n, uint64_t n_acc_total) {
     if ((n.par_dims != 1 && n.par_dims != 2) || n.depth > 3 || (n.par_dims == 1 && n.P1 != 1) ||
         uint64_t(n.access_off) + uint64_t(n.n_access) > n_acc_total)
         return SEL_EINVAL;
     const uint64_t P = smul(n.P0, n.P1);
     if (n.P0 >= kLim40 || P >= kLim40) return SEL_ERANGE;
+    return SEL_OK;
+}
+// P = P0 P1, T = effective trips of the nest
+__device__ __forceinline__ uint32_t access_check(const sel_access& a, uint32_t par_dims, uint32_t depth, uint64_t P,
+                                                 uint64_t P0, uint64_t P1, const uint64_t T[3], uint64_t* Mk_out) {
+    const int64_t e = a.elem_bytes;
+    if (!(e == 1 || e == 2 || e == 4 || e == 8 || e == 16) || a.depth > depth) return kAccInval;
+    // power-of-two element size: divisibility by masking
+    const int64_t m = e - 1;
+    bool bad = (a.base & m) || (a.c_par[0] & m) || (par_dims == 2 && (a.c_par[1] & m));
+    for (int j = 0; j < a.depth; j++) bad |= (a.c_inner[j] & m) != 0;
+    if (bad) return kAccInval;
+    const uint64_t e0 = (par_dims == 1) ? P : P0;
+    uint64_t bound = uabs(a.base);
+    bound = sadd(bound, smul(uabs(a.c_par[0]), e0 ? e0 - 1 : 0));
+    if (par_dims == 2) bound = sadd(bound, smul(uabs(a.c_par[1]), P1 ? P1 - 1 : 0));
+    uint64_t Mk = 1;
+    for (int j = 0; j < a.depth; j++) {
+        bound = sadd(bound, smul(uabs(a.c_inner[j]), T[j] ? T[j] - 1 : 0));
+        Mk = smul(Mk, T[j]);
+    }
+    *Mk_out = Mk;
+    return bound >= kLim62 ? kAccRange : 0u;
+}
+__device__ __forceinline__ uint8_t nest_status(uint8_t pre, uint32_t acc_flags, uint64_t P, uint64_t M_it) {
+    if (pre) return pre;
+    if (acc_flags & kAccInval) return SEL_EINVAL;
+    if (acc_flags & kAccRange) return SEL_ERANGE;
+    if (smul(P, M_it) >= kLim48) return SEL_ERANGE;
+    return SEL_OK;
+}
+
+// Nest-level checks V3-V6; on success *M_it = sum_k prod_{j<depth_k} T_j.
+__device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc_all, uint64_t n_acc_total,
+                                        uint64_t* M_it_out) {
+    const uint8_t pre = nest_precheck(n, n_acc_total);
+    if (pre) return pre;
+    const uint64_t P = smul(n.P0, n.P1);
     uint64_t T[3];
     for (int j = 0; j < 3; j++) T[j] = eff_trip(n.trip[j]);
     const sel_access* acc = acc_all + n.access_off;
-    for (uint32_t k = 0; k < n.n_access; k++) {
-        const sel_access a = acc[k];
-        const int64_t e = a.elem_bytes;
-        if (!(e == 1 || e == 2 || e == 4 || e == 8 || e == 16) || a.depth > n.depth) return SEL_EINVAL;
-        // power-of-two element size: divisibility by masking
-        const int64_t m = e - 1;
-        bool bad = (a.base & m) || (a.c_par[0] & m) || (n.par_dims == 2 && (a.c_par[1] & m));
-        for (int j = 0; j < a.depth; j++) bad |= (a.c_inner[j] & m) != 0;
-        if (bad) return SEL_EINVAL;
-    }
+    uint32_t flags = 0;
     uint64_t M_it = 0;
     for (uint32_t k = 0; k < n.n_access; k++) {
-        const sel_access a = acc[k];
-        const uint64_t e0 = (n.par_dims == 1) ? P : n.P0;
-        uint64_t bound = uabs(a.base);
-        bound = sadd(bound, smul(uabs(a.c_par[0]), e0 ? e0 - 1 : 0));
-        if (n.par_dims == 2) bound = sadd(bound, smul(uabs(a.c_par[1]), n.P1 ? n.P1 - 1 : 0));
-        uint64_t Mk = 1;
-        for (int j = 0; j < a.depth; j++) {
-            bound = sadd(bound, smul(uabs(a.c_inner[j]), T[j] ? T[j] - 1 : 0));
-            Mk = smul(Mk, T[j]);
-        }
-        if (bound >= kLim62) return SEL_ERANGE;
+        uint64_t Mk = 0;
+        flags |= access_check(acc[k], n.par_dims, n.depth, P, n.P0, n.P1, T, &Mk);
+        if (flags & kAccInval) break;
         M_it = sadd(M_it, Mk);
     }
-    if (smul(P, M_it) >= kLim48) return SEL_ERANGE;
-    *M_it_out = M_it;
-    return SEL_OK;
+    const uint8_t st = nest_status(SEL_OK, flags, P, M_it);
+    if (st == SEL_OK) *M_it_out = M_it;
+    return st;
 }
 
 // Problems counted one per lane (k_lane_problems) rather than through the WA

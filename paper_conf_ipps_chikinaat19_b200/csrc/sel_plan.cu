@@ -317,28 +317,97 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
     const uint64_t nq = hdr->n_problems;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     if (hdr->direct) {
-        // direct ids: the problems of nest i are i * n_cls + [0, n_cls) -- one thread
-        // per nest validates it once for all of them
+        // direct ids: the problems of nest i are i * n_cls + [0, n_cls).  A warp
+        // takes 32 nests (lane = nest), checks the concatenation of their access
+        // lists 32 accesses at a time (lane = access: the descriptor loads are
+        // independent and, for consecutive nests, contiguous), reduces each
+        // nest's flags and M_it (saturating) over its lanes, and the nest's lane
+        // writes its n_cls problems.
+        __shared__ uint32_t s_flags[8][32];
+        __shared__ unsigned long long s_mit[8][32];
         const uint32_t ncls = hdr->n_cls;
         const uint64_t nn = ncls ? nq / ncls : 0;
+        const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+        const uint64_t nwarps = uint64_t(gridDim.x) * (blockDim.x >> 5);
         uint32_t used = 0;
-        for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < nn; i += stride) {
+        for (uint64_t i0 = (uint64_t(blockIdx.x) * (blockDim.x >> 5) + wib) * 32; i0 < nn; i0 += nwarps * 32) {
+            const uint64_t i = i0 + lane;
             uint32_t um = 0;
-            for (uint32_t c = 0; c < ncls; c++) um |= (prob_nest[i * ncls + c] != kNoProblem ? 1u : 0u) << (c & 31u);
             sel_nest nest{};
-            uint64_t M_it = 0;
-            uint8_t st = SEL_EINVAL;
-            if (um) {
-                nest = t.nests[i];
-                st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
+            uint8_t pre = SEL_EINVAL;
+            if (i < nn) {
+                for (uint32_t c = 0; c < ncls; c++) um |= (prob_nest[i * ncls + c] != kNoProblem ? 1u : 0u) << (c & 31u);
+                if (um || ncls > 32) {
+                    nest = t.nests[i];
+                    pre = nest_precheck(nest, t.n_accesses);
+                }
             }
-            for (uint32_t c = 0; c < ncls; c++) {
-                const uint64_t q = i * ncls + c;
-                const bool u = c < 32 ? ((um >> c) & 1u) : prob_nest[q] != kNoProblem;
-                used += u ? 1u : 0u;
-                problem_w_one(q, nest, u ? st : uint8_t(SEL_EINVAL), M_it, prob_B, prob_W, prob_WR, prob_status,
-                              prob_cnt, lane_ok);
+            const uint32_t na = pre == SEL_OK ? nest.n_access : 0u;
+            uint32_t incl = na;                                 // inclusive prefix of the access counts
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
             }
+            const uint32_t tot = __shfl_sync(kFull, incl, 31);
+            const uint64_t P = smul(nest.P0, nest.P1);
+            s_flags[wib][lane] = 0u;
+            s_mit[wib][lane] = 0ull;
+            __syncwarp();
+            for (uint32_t j0 = 0; j0 < tot; j0 += 32) {
+                const uint32_t j = j0 + uint32_t(lane);
+                // owner: the first lane whose inclusive prefix exceeds j
+                int own = 0;
+#pragma unroll
+                for (int step = 16; step; step >>= 1) {
+                    const uint32_t v = __shfl_sync(kFull, incl, own + step - 1);
+                    if (v <= j) own += step;
+                }
+                own = own > 31 ? 31 : own;
+                const uint32_t ex = __shfl_sync(kFull, incl - na, own);
+                const uint32_t aoff = __shfl_sync(kFull, nest.access_off, own);
+                const uint32_t pd = __shfl_sync(kFull, uint32_t(nest.par_dims), own);
+                const uint32_t dp = __shfl_sync(kFull, uint32_t(nest.depth), own);
+                const uint64_t Po = __shfl_sync(kFull, P, own), P0o = __shfl_sync(kFull, nest.P0, own),
+                               P1o = __shfl_sync(kFull, nest.P1, own);
+                const uint64_t T[3] = {eff_trip(__shfl_sync(kFull, nest.trip[0], own)),
+                                       eff_trip(__shfl_sync(kFull, nest.trip[1], own)),
+                                       eff_trip(__shfl_sync(kFull, nest.trip[2], own))};
+                uint32_t fl = 0;
+                uint64_t Mk = 0;
+                if (j < tot) fl = access_check(t.accesses[aoff + (j - ex)], pd, dp, Po, P0o, P1o, T, &Mk);
+                // segmented (by owner) saturating sum over the lanes of this round
+                const bool in = j < tot;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint64_t y = __shfl_up_sync(kFull, Mk, o);
+                    const uint32_t yf = __shfl_up_sync(kFull, fl, o);
+                    const int yo = __shfl_up_sync(kFull, own, o);
+                    if (lane >= o && yo == own) {
+                        Mk = sadd(Mk, y);
+                        fl |= yf;
+                    }
+                }
+                const int nxt = __shfl_down_sync(kFull, own, 1);
+                const bool tail = in && (lane == 31 || j + 1 >= tot || nxt != own);
+                if (tail) {                                     // one lane per owner per round
+                    s_mit[wib][own] = sadd(s_mit[wib][own], Mk);
+                    s_flags[wib][own] |= fl;
+                }
+                __syncwarp();
+            }
+            if (i < nn) {
+                const uint64_t M_it = s_mit[wib][lane];
+                const uint8_t st = nest_status(pre, s_flags[wib][lane], P, M_it);
+                for (uint32_t c = 0; c < ncls; c++) {
+                    const uint64_t q = i * ncls + c;
+                    const bool u = c < 32 ? ((um >> c) & 1u) : prob_nest[q] != kNoProblem;
+                    used += u ? 1u : 0u;
+                    problem_w_one(q, nest, u ? st : uint8_t(SEL_EINVAL), st == SEL_OK ? M_it : 0ull, prob_B, prob_W,
+                                  prob_WR, prob_status, prob_cnt, lane_ok);
+                }
+            }
+            __syncwarp();
         }
         used = __reduce_add_sync(kFull, used);
         if ((threadIdx.x & 31) == 0 && used) atomicAdd((unsigned long long*)&hdr->stats.n_problems, (unsigned long long)used);

@@ -34,6 +34,8 @@ WORKLOAD = ("c5: 10^8-candidate selection sweep (24 Polybench-shaped nests x tri
             "8 launch configs x 4 device sets)")
 OPS_PER_WA = 224           # 7 integer lane-ops x 32 lanes per warp-access (lane expansion)
 CAND_BYTES = 24 + 1 + 8    # per candidate: sel_candidate read, decision + cycles written
+MODEL_BYTES = 24 + 1 + 8 + 1   # model kernels: record in, decision + cycles + status out
+PLAN_BYTES = 24 + 4 + 1    # plan: record in, problem id + candidate status out
 
 
 def parse():
@@ -118,28 +120,34 @@ def measured_peaks():
         return {}
 
 
-def ncu_capture():
-    """Counters of the committed ncu --set full capture of the counting kernel
-    in this bench configuration (profiles/ncu_count_kernel.json)."""
+NCU_REGION_KERNELS = {
+    "plan": ("k_classes", "k_insert", "k_rank_slots", "k_scan_reduce", "k_scan_partials", "k_scan_down", "k_assign",
+             "k_finalize_plan", "k_problem_w", "k_plan_stats"),
+    "count": ("k_lane_problems", "k_queue", "k_count"),
+    "model": ("k_problem_model", "k_model_fused"),
+}
+
+
+def ncu_kernels():
+    """Per-kernel counters of the committed ncu --set full capture of one bench
+    step (profiles/ncu_kernels.json, written by scripts/ncu_kernels.py)."""
     try:
-        with open(os.path.join(ROOT, "profiles", "ncu_count_kernel.json")) as f:
-            d = json.load(f)
+        with open(os.path.join(ROOT, "profiles", "ncu_kernels.json")) as f:
+            return json.load(f)
     except (OSError, ValueError):
         return {}
-    k = d.get("count_kernel_full", {})
-    out = {"traffic": d.get("dram_bytes_per_launch"),
-           "warp_instructions_per_wa": d.get("warp_instructions_per_wa")}
-    for key, name in (("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "alu_pipe_pct"),
-                      ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "fma_pipe_pct"),
-                      ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue_active_pct")):
-        if key in k:
-            out[name] = k[key]
-    return out
 
 
-def ncu_traffic_per_launch():
-    """dram bytes per counting-kernel launch from the committed ncu capture."""
-    return ncu_capture().get("traffic")
+def ncu_region_traffic(ncu, region):
+    """dram read + write bytes per launch of a region's kernels (committed capture), or None."""
+    ks = [ncu["kernels"][k] for k in NCU_REGION_KERNELS[region] if k in ncu.get("kernels", {})]
+    return sum(k["dram_bytes"] for k in ks) if ks else None
+
+
+def ncu_region(ncu, region):
+    """The committed capture's counters of the region's kernels (source: profiles/ncu_kernels.json)."""
+    ks = {k: v for k, v in ncu.get("kernels", {}).items() if k in NCU_REGION_KERNELS[region]}
+    return {"source": ncu.get("source"), "kernels": ks} if ks else {}
 
 
 def cpu_oracle_sample(batch, seconds: float, total_candidates: int):
@@ -250,7 +258,8 @@ def run_ours(args):
     torch.cuda.synchronize(dev)
     stats = ev.stats()
     sel.profile_enable(True)
-    sel.profile_read()
+    for r in (sel.PROF_PLAN, sel.PROF_COUNT, sel.PROF_MODEL):
+        sel.profile_read_region(r)
     launches0 = sel.kernel_launches()
     D.barrier(world)
     torch.cuda.synchronize(dev)
@@ -264,7 +273,9 @@ def run_ours(args):
     D.barrier(world)
     ms_local = e0.elapsed_time(e1)
     launches = sel.kernel_launches() - launches0
-    count_ms, count_launches = sel.profile_read()
+    plan_ms, plan_launches = sel.profile_read_region(sel.PROF_PLAN)
+    count_ms, count_launches = sel.profile_read_region(sel.PROF_COUNT)
+    model_ms, model_launches = sel.profile_read_region(sel.PROF_MODEL)
     sel.profile_enable(False)
     ms = D.max_over_ranks(ms_local, world, dev)
     wa_analysed = D.sum_over_ranks(stats["wa_analysed"], world, dev)
@@ -304,42 +315,65 @@ def run_ours(args):
 
     if rank != 0:
         return
-    # ---- roofline of the counting kernels (INT bound): peak = measured INT32 lane-op
-    # rate with the ALU and FMA pipes both issuing (sel_int_peak mode 2), all SMs.  achieved = the
-    # nominal algorithmic lane-ops the counting kernels performed (sel_stats.alg_lane_ops: 224 per
-    # expanded WA, 12 per arithmetic-lane WA, 6 per uniform class, 6 / 5 / 12 per histogram entry /
-    # convolution term / residue evaluation) / their measured time (CUDA events on the launching stream)
+    # ---- per-region device time (CUDA events the library records on the launching stream around the
+    # plan, counting and model kernels of every call) and the roofline of each
     f_mhz = clocks["sm_mhz"] or measured_peaks().get("clocks_under_load", {}).get("sm_mhz_median", 1965.0)
+    hbm_peak = measured_peaks().get("hbm_gbs")
+    ncu = ncu_kernels()
+    per_launch = {"plan": plan_ms / max(plan_launches, 1), "count": count_ms / max(count_launches, 1),
+                  "model": model_ms / max(model_launches, 1)}
+    # counting kernels: INT bound.  peak = measured INT32 lane-op rate with the ALU and FMA pipes both
+    # issuing (sel_int_peak mode 2), all SMs.  achieved = the nominal algorithmic lane-ops of the paths
+    # the counting kernels took (sel_stats.alg_lane_ops) / their measured time
     peak_ops = int_peak["both"]
     wa_arith, wa_res, wa_cf = stats["wa_arith_lanes"], stats["wa_residue_classes"], stats["wa_closed_form"]
     wa_lane = stats["wa_analysed"] - wa_cf - wa_arith - wa_res
-    avg_count_ms = count_ms / max(count_launches, 1)
+    avg_count_ms = per_launch["count"]
     achieved = stats["alg_lane_ops"] / (avg_count_ms / 1e3)
     survey_eq = stats["wa_analysed"] * OPS_PER_WA / (avg_count_ms / 1e3)
-    roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
-                "frac": achieved / peak_ops, "traffic": ncu_traffic_per_launch(),
-                "kernel": "counting kernels (k_lane_problems + k_queue + k_count)",
-                "count_ms_per_launch": avg_count_ms, "count_share_of_step": avg_count_ms / (t_step * 1e3),
-                "alg_lane_ops_per_step": stats["alg_lane_ops"],
-                "peak_source": "measured: sel_int_peak (independent IADD3/LOP3 + IMAD chains, all SMs, ALU and FMA "
-                               "pipes both issuing) at the run's clocks",
-                "peak_alu_pipe_only": int_peak["alu"] / 1e12, "peak_fma_pipe_only": int_peak["fma"] / 1e12,
-                "peak_nominal_issue": 148 * 128 * f_mhz * 1e6 / 1e12,
-                "wa_per_path": {"lane_expansion": wa_lane, "arith_lanes": wa_arith, "residue_classes": wa_res,
-                                "uniform_closed_form": wa_cf},
-                "survey_equivalent": {"ops_per_wa": OPS_PER_WA, "achieved": survey_eq / 1e12,
-                                      "ratio_to_peak": survey_eq / peak_ops,
-                                      "note": "SURVEY §8(d)'s 224 lane-ops x every analysed warp-access / counting "
-                                              "time: the brute-force expansion rate the exact closed forms stand "
-                                              "in for (> 1 = faster than expanding at the INT peak)"},
-                "note": ("achieved = nominal algorithmic lane-ops of the paths the counting kernels took "
-                         "(sel_stats.alg_lane_ops) / their time; ncu_* are the issued-instruction counters of the "
-                         "committed capture"),
-                "ncu": ncu_capture()}
+    roof_count = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
+                  "frac": achieved / peak_ops, "traffic": ncu_region_traffic(ncu, "count"),
+                  "kernel": "counting kernels (k_lane_problems + k_queue + k_count)",
+                  "ms_per_launch": avg_count_ms, "share_of_step": avg_count_ms / (t_step * 1e3),
+                  "alg_lane_ops_per_step": stats["alg_lane_ops"],
+                  "peak_source": "measured: sel_int_peak (independent IADD3/LOP3 + IMAD chains, all SMs, ALU and "
+                                 "FMA pipes both issuing) at the run's clocks",
+                  "peak_alu_pipe_only": int_peak["alu"] / 1e12, "peak_fma_pipe_only": int_peak["fma"] / 1e12,
+                  "peak_nominal_issue": 148 * 128 * f_mhz * 1e6 / 1e12,
+                  "wa_per_path": {"lane_expansion": wa_lane, "arith_lanes": wa_arith, "residue_classes": wa_res,
+                                  "uniform_closed_form": wa_cf},
+                  "survey_equivalent": {"ops_per_wa": OPS_PER_WA, "achieved": survey_eq / 1e12,
+                                        "ratio_to_peak": survey_eq / peak_ops,
+                                        "note": "SURVEY §8(d)'s 224 lane-ops x every analysed warp-access / "
+                                                "counting time: the brute-force expansion rate the exact closed "
+                                                "forms stand in for (> 1 = faster than expanding at the INT peak)"},
+                  "note": ("achieved = nominal algorithmic lane-ops of the paths the counting kernels took "
+                           "(sel_stats.alg_lane_ops) / their time"),
+                  "ncu": ncu_region(ncu, "count")}
+    # model kernels (k_problem_model + k_model_fused): per candidate the 24 B record in, decision (1) +
+    # cycles (8) + status (1) out -- HBM is the roofline of a streaming per-candidate kernel
+    def hbm_roof(name, kernel, bytes_per_launch, detail):
+        ms = per_launch[name]
+        a = bytes_per_launch / (ms / 1e3) / 1e9 if ms > 0 else 0.0
+        r = {"bound": "hbm", "achieved": a, "peak": hbm_peak, "unit": "GB/s",
+             "frac": a / hbm_peak if hbm_peak else None, "traffic": ncu_region_traffic(ncu, name),
+             "kernel": kernel, "ms_per_launch": ms, "share_of_step": ms / (t_step * 1e3),
+             "algorithmic_bytes_per_launch": bytes_per_launch, "bytes": detail,
+             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth, burst)", "ncu": ncu_region(ncu, name)}
+        return r
+    n_nests, n_acc = len(batch.nests), len(batch.accesses)
+    roof_model = hbm_roof("model", "model kernels (k_problem_model + k_model_fused)", MODEL_BYTES * len(batch),
+                          f"{MODEL_BYTES} B per candidate (record in, decision + cycles + status out)")
+    roof_plan = hbm_roof("plan", "plan kernels (k_classes, k_insert, k_problem_w, scans, ...)",
+                         PLAN_BYTES * len(batch) + 88 * n_nests + 64 * n_acc,
+                         f"{PLAN_BYTES} B per candidate (record in, problem id + status out) + every nest (88 B) "
+                         f"and access (64 B) record once")
+    regions = {"plan": roof_plan, "count": roof_count, "model": roof_model}
+    dominant = max(per_launch, key=per_launch.get)
+    roofline = dict(regions[dominant], region=dominant)
     # the whole step against HBM: per candidate the 24 B record in, decision + cycles out
     step_hbm = {"bound": "hbm", "bytes_per_candidate": CAND_BYTES,
-                "achieved": CAND_BYTES * total / t_step / 1e9, "peak": measured_peaks().get("hbm_gbs"),
-                "unit": "GB/s"}
+                "achieved": CAND_BYTES * total / t_step / 1e9, "peak": hbm_peak, "unit": "GB/s"}
     if step_hbm["peak"]:
         step_hbm["frac"] = step_hbm["achieved"] / step_hbm["peak"]
     hbm_bytes = (24 + 9) * total                     # candidate read + decision/cycles write per step
@@ -361,7 +395,11 @@ def run_ours(args):
             "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
             "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
             "wa_closed_form_per_step": wa_closed,
-            "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline, "step_hbm_roofline": step_hbm,
+            "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline,
+            "roofline_by_region": {k: {kk: v[kk] for kk in ("bound", "achieved", "peak", "unit", "frac", "traffic",
+                                                            "ms_per_launch", "share_of_step")}
+                                   for k, v in regions.items()},
+            "roofline_count": roof_count, "step_hbm_roofline": step_hbm,
             "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
     if not args.no_next and args.config == 5:

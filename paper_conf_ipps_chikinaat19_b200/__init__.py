@@ -23,7 +23,7 @@ from ._lib import (DECISION_CPU, DECISION_GPU, DECISION_INVALID, SEL_EINTERNAL, 
                    SEL_ERANGE, SEL_F_MATCH_ANY, SEL_F_NO_DEDUP, SEL_OK, SelError)
 
 __all__ = ["load_device_params", "workspace_size", "DeviceTables", "count_transactions", "predict_gpu_cycles",
-           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "kernel_launches",
+           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "profile_read_region", "PROF_PLAN", "PROF_COUNT", "PROF_MODEL", "kernel_launches",
            "Evaluator", "SelError", "SEL_F_NO_DEDUP", "SEL_F_MATCH_ANY", "DECISION_CPU", "DECISION_GPU",
            "DECISION_INVALID", "SEL_OK", "SEL_EINVAL", "SEL_ERANGE", "SEL_ELAUNCH", "SEL_EINTERNAL"]
 
@@ -230,6 +230,17 @@ def profile_read():
     """-> (counting-kernel milliseconds, counting launches) since the last read."""
     ms, k = ctypes.c_double(), ctypes.c_uint64()
     _lib.check(_lib.lib().sel_profile_read(ctypes.byref(ms), ctypes.byref(k)))
+    return ms.value, k.value
+
+
+PROF_PLAN, PROF_COUNT, PROF_MODEL = 0, 1, 2        # sel.h SEL_PROF_*
+
+
+def profile_read_region(region: int):
+    """-> (milliseconds, launches) of one profiling region (PROF_PLAN,
+    PROF_COUNT, PROF_MODEL) since its last read."""
+    ms, k = ctypes.c_double(), ctypes.c_uint64()
+    _lib.check(_lib.lib().sel_profile_read_region(int(region), ctypes.byref(ms), ctypes.byref(k)))
     return ms.value, k.value
 
 

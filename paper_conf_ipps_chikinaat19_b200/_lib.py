@@ -110,6 +110,8 @@ def lib():
         L.sel_bind_accesses.argtypes = [vp, u64, vp, u64, vp, u64, vp, u64, vp, vp, vp]
         L.sel_profile_enable.argtypes = [ctypes.c_int]
         L.sel_profile_read.argtypes = [ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64)]
+        L.sel_profile_read_region.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_double),
+                                              ctypes.POINTER(ctypes.c_uint64)]
         L.sel_kernel_launches.restype = u64
         L.sel_int_peak.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_double)]
         L.sel_last_error.restype = ctypes.c_char_p
@@ -132,5 +134,5 @@ def check(rc: int):
 
 EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions", "sel_count_transactions_part",
             "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_select_launch", "sel_model_cpu_cost", "sel_bind_accesses", "sel_read_stats",
-            "sel_profile_enable", "sel_profile_read", "sel_kernel_launches", "sel_int_peak", "sel_last_error",
+            "sel_profile_enable", "sel_profile_read", "sel_profile_read_region", "sel_kernel_launches", "sel_int_peak", "sel_last_error",
             "sel_version", "sel_sizeof", "sel_offsetof")

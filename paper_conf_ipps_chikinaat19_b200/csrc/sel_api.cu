@@ -27,11 +27,13 @@ static int cuda_fail(cudaError_t e, const char* where) {
 }
 
 // ------------------------------------------------------------- profiling
+// Regions (sel.h SEL_PROF_*): CUDA events recorded on the launching stream
+// around the plan, counting and model kernels of every call.
 static std::mutex g_prof_mu;
 static bool g_prof_on = false;
-static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_prof_pending;
+static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_prof_pending[SEL_PROF_REGIONS];
 static std::vector<cudaEvent_t> g_prof_free;
-static cudaEvent_t g_prof_cur_begin = nullptr;
+static cudaEvent_t g_prof_cur_begin[SEL_PROF_REGIONS] = {};
 
 static cudaEvent_t prof_event() {
     if (!g_prof_free.empty()) {
@@ -44,20 +46,22 @@ static cudaEvent_t prof_event() {
     return e;
 }
 
-void prof_before_count(cudaStream_t s) {
+void prof_begin(int region, cudaStream_t s) {
     std::lock_guard<std::mutex> g(g_prof_mu);
     if (!g_prof_on) return;
-    g_prof_cur_begin = prof_event();
-    cudaEventRecord(g_prof_cur_begin, s);
+    g_prof_cur_begin[region] = prof_event();
+    cudaEventRecord(g_prof_cur_begin[region], s);
 }
-void prof_after_count(cudaStream_t s) {
+void prof_end(int region, cudaStream_t s) {
     std::lock_guard<std::mutex> g(g_prof_mu);
-    if (!g_prof_on || !g_prof_cur_begin) return;
+    if (!g_prof_on || !g_prof_cur_begin[region]) return;
     cudaEvent_t e = prof_event();
     cudaEventRecord(e, s);
-    g_prof_pending.emplace_back(g_prof_cur_begin, e);
-    g_prof_cur_begin = nullptr;
+    g_prof_pending[region].emplace_back(g_prof_cur_begin[region], e);
+    g_prof_cur_begin[region] = nullptr;
 }
+void prof_before_count(cudaStream_t s) { prof_begin(SEL_PROF_COUNT, s); }
+void prof_after_count(cudaStream_t s) { prof_end(SEL_PROF_COUNT, s); }
 
 WsPtrs ws_ptrs(void* ws, uint64_t n, uint64_t n_nests, uint32_t flags) {
     const WsLayout L = ws_layout(n, n_nests, flags);
@@ -247,11 +251,12 @@ int sel_profile_enable(int on) {
     return SEL_OK;
 }
 
-int sel_profile_read(double* count_ms, uint64_t* count_launches) {
+int sel_profile_read_region(int region, double* ms_out, uint64_t* launches_out) {
+    if (region < 0 || region >= SEL_PROF_REGIONS) return fail(SEL_EINVAL, "unknown profiling region%s");
     std::lock_guard<std::mutex> g(g_prof_mu);
     double ms = 0.0;
     uint64_t k = 0;
-    for (auto& pr : g_prof_pending) {
+    for (auto& pr : g_prof_pending[region]) {
         cudaError_t e = cudaEventSynchronize(pr.second);
         if (e != cudaSuccess) return cuda_fail(e, "sel_profile_read");
         float x = 0.f;
@@ -261,10 +266,14 @@ int sel_profile_read(double* count_ms, uint64_t* count_launches) {
         g_prof_free.push_back(pr.first);
         g_prof_free.push_back(pr.second);
     }
-    g_prof_pending.clear();
-    if (count_ms) *count_ms = ms;
-    if (count_launches) *count_launches = k;
+    g_prof_pending[region].clear();
+    if (ms_out) *ms_out = ms;
+    if (launches_out) *launches_out = k;
     return SEL_OK;
+}
+
+int sel_profile_read(double* count_ms, uint64_t* count_launches) {
+    return sel_profile_read_region(SEL_PROF_COUNT, count_ms, count_launches);
 }
 
 uint64_t sel_kernel_launches(void) { return g_launches.load(); }

@@ -34,6 +34,8 @@ void note_launch(int k = 1);
 // records the profiling events around the counting kernel, when enabled
 void prof_before_count(cudaStream_t s);
 void prof_after_count(cudaStream_t s);
+void prof_begin(int region, cudaStream_t s);
+void prof_end(int region, cudaStream_t s);
 
 // sel_plan.cu: candidates -> counting problems, closed-form W per problem, prefix
 cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables& t, int n_sets,

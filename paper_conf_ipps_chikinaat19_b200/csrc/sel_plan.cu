@@ -448,6 +448,7 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
                         const WsPtrs& w, uint64_t n_nests, uint32_t flags, uint32_t part, uint32_t n_parts,
                         cudaStream_t s) {
     const bool dedup = !(flags & SEL_F_NO_DEDUP);
+    prof_begin(SEL_PROF_PLAN, s);
     cudaError_t e = cudaMemsetAsync(w.hdr, 0, sizeof(WsHeader), s);
     if (e != cudaSuccess) return e;
     if (dedup && n_nests) {
@@ -482,6 +483,7 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
     if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s)) != cudaSuccess) return e;
     k_plan_stats<<<1, 1, 0, s>>>(w.hdr, w.prob_W);
     note_launch();
+    prof_end(SEL_PROF_PLAN, s);
     return cudaGetLastError();
 }
 

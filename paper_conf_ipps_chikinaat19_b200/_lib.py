@@ -114,6 +114,8 @@ def lib():
                                               ctypes.POINTER(ctypes.c_uint64)]
         L.sel_kernel_launches.restype = u64
         L.sel_int_peak.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_double)]
+        L.sel_selftest_ddiv.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p,
+                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
         L.sel_last_error.restype = ctypes.c_char_p
         L.sel_version.restype = ctypes.c_char_p
         L.sel_sizeof.restype = sz
@@ -134,5 +136,5 @@ def check(rc: int):
 
 EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions", "sel_count_transactions_part",
             "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_select_launch", "sel_model_cpu_cost", "sel_bind_accesses", "sel_read_stats",
-            "sel_profile_enable", "sel_profile_read", "sel_profile_read_region", "sel_kernel_launches", "sel_int_peak", "sel_last_error",
+            "sel_profile_enable", "sel_profile_read", "sel_profile_read_region", "sel_kernel_launches", "sel_int_peak", "sel_selftest_ddiv", "sel_last_error",
             "sel_version", "sel_sizeof", "sel_offsetof")

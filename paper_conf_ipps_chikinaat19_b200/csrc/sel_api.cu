@@ -278,6 +278,14 @@ int sel_profile_read(double* count_ms, uint64_t* count_launches) {
 
 uint64_t sel_kernel_launches(void) { return g_launches.load(); }
 
+int sel_selftest_ddiv(const double* a, const double* b, uint64_t n, double* q_fast, uint8_t* ok, double* q_ref,
+                      sel_stream_t stream) {
+    if (n && (!a || !b || !q_fast || !ok || !q_ref)) return fail(SEL_EINVAL, "NULL argument%s");
+    cudaError_t e = launch_selftest_ddiv(a, b, n, q_fast, ok, q_ref, reinterpret_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "sel_selftest_ddiv");
+    return SEL_OK;
+}
+
 const char* sel_last_error(void) { return t_err; }
 const char* sel_version(void) { return "libsel 0.1 sm_100a"; }
 

@@ -55,6 +55,8 @@ cudaError_t launch_model_fused(const sel_candidate* cands, uint64_t n, const sel
 cudaError_t launch_model_from_counts(const sel_candidate* cands, uint64_t n, const sel_tables& t,
                                      const sel_counts* counts, double* cycles, double* t_gpu, uint8_t* status,
                                      cudaStream_t s);
+cudaError_t launch_selftest_ddiv(const double* a, const double* b, uint64_t n, double* q_fast, uint8_t* ok,
+                                 double* q_ref, cudaStream_t s);
 cudaError_t launch_select(const sel_candidate* cands, uint64_t n, const double* t_gpu, const uint8_t* status,
                           uint8_t* decision, cudaStream_t s);
 

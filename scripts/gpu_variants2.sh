@@ -12,5 +12,5 @@ for v in $VARIANTS; do
   SEL_LIBSEL=/tmp/libsel_$name.so timeout 600 python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline --no-next > gpurun_out/bench_$name.json 2>> gpurun_out/bench.err
 done
 tail -3 gpurun_out/tests.log
-for f in gpurun_out/bench*.json; do python -c "import json,sys; d=json.loads(open('$f').read()); print('$f', 'G/s', round(d['value']/1e9,3), 'ms', round(d['ms_per_step'],3), 'count_ms', round(d['roofline']['count_ms_per_launch'],3))"; done
+for f in gpurun_out/bench*.json; do python -c "import json,sys; d=json.loads(open('$f').read()); print('$f', 'G/s', round(d['value']/1e9,3), 'ms', round(d['ms_per_step'],3), {k: round(v['ms_per_launch'],3) for k, v in d['roofline_by_region'].items()})"; done
 tail -3 gpurun_out/bench.err

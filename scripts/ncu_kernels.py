@@ -54,7 +54,8 @@ def main():
                 continue
             u = units[i]
             if short == "time_ms":
-                v *= {"second": 1e3, "msecond": 1.0, "usecond": 1e-3, "nsecond": 1e-6}.get(u, 1.0)
+                v *= {"second": 1e3, "s": 1e3, "msecond": 1.0, "ms": 1.0, "usecond": 1e-3, "us": 1e-3,
+                      "nsecond": 1e-6, "ns": 1e-6}.get(u, 1.0)
             elif short.startswith("dram_") and short != "dram_throughput_pct":
                 v *= UNIT.get(u, 1.0)
             d[short] = v

@@ -1395,9 +1395,13 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
 #endif
 constexpr uint32_t kLaneGrp = 4;        // problems of a unit counted together
 constexpr uint32_t kLaneTile = 2048;    // units sorted per block tile
-constexpr uint32_t kLaneKeys = 256;
+constexpr uint32_t kLaneKeyBits = 8;
+constexpr uint32_t kLaneKeys = 1u << kLaneKeyBits;
 constexpr size_t kLaneSmem = (size_t(kLaneRows) * kLaneThreads + kLaneTile + kLaneKeys) * sizeof(uint32_t);
 
+// shape key of a unit: accesses, loop depth, collapse (keys that also hash the
+// first accesses' counting paths and element sizes cost more in descriptor loads
+// than they gained in SIMT efficiency: profiles/r01_variants_v8/)
 __device__ __forceinline__ uint32_t lane_unit_key(const CountArgs& a, uint64_t u, bool direct) {
     const uint32_t nid = direct ? uint32_t(u) : a.prob_nest[u];
     if (nid == kNoProblem) return 0u;

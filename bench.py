@@ -57,6 +57,11 @@ def parse():
 
 # ---------------------------------------------------------------- clocks
 class ClockSampler:
+    """SM clock and throttle reasons sampled DURING the timed region: an NVML
+    polling thread (every ~2 ms, so a region of a few tens of ms still gets
+    samples), falling back to `nvidia-smi -lms`."""
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4))
     FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
               "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
@@ -65,8 +70,34 @@ class ClockSampler:
         self.idx = gpu_index
         self.proc = None
         self.lines = []
+        self.samples = []               # (sm_mhz, max_mhz, reason bits) from NVML
+        self.nvml = None
+        self.stop = threading.Event()
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        try:
+            import torch
+            bus = torch.cuda.get_device_properties(self.idx).pci_bus_id
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId_v2(
+                "%08x:%02x:%02x.0" % (torch.cuda.get_device_properties(self.idx).pci_domain_id, bus,
+                                      torch.cuda.get_device_properties(self.idx).pci_device_id))
+        except Exception:
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            idx = int(vis.split(",")[self.idx]) if vis and vis.split(",")[self.idx].isdigit() else self.idx
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(idx)
 
     def __enter__(self):
+        try:
+            self.nvml = self._nvml_handle()
+            pm, h = self.nvml
+            self.max_mhz = float(pm.nvmlDeviceGetMaxClockInfo(h, pm.NVML_CLOCK_SM))
+            self.t = threading.Thread(target=self._poll, daemon=True)
+            self.t.start()
+            return self
+        except Exception:
+            self.nvml = None
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.FIELDS}",
                                           "--format=csv,noheader,nounits", "-lms", "200"],
@@ -77,11 +108,24 @@ class ClockSampler:
             self.proc = None
         return self
 
+    def _poll(self):
+        pm, h = self.nvml
+        while not self.stop.is_set():
+            try:
+                self.samples.append((float(pm.nvmlDeviceGetClockInfo(h, pm.NVML_CLOCK_SM)), self.max_mhz,
+                                     int(pm.nvmlDeviceGetCurrentClocksEventReasons(h))))
+            except Exception:
+                pass
+            self.stop.wait(0.002)
+
     def _read(self):
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
     def __exit__(self, *a):
+        self.stop.set()
+        if self.nvml:
+            self.t.join(timeout=2)
         if self.proc:
             self.proc.terminate()
             try:
@@ -92,6 +136,12 @@ class ClockSampler:
 
     def summary(self):
         sm, smax, reasons = [], 0.0, set()
+        for mhz, mx, bits in self.samples:
+            sm.append(mhz)
+            smax = max(smax, mx)
+            for name, bit in self.REASONS:
+                if bits & bit:
+                    reasons.add(name)
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
             f = [x.strip() for x in ln.split(",")]
@@ -108,7 +158,7 @@ class ClockSampler:
         if not sm:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
         return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons),
-                "samples": len(sm)}
+                "samples": len(sm), "source": "nvml" if self.samples else "nvidia-smi"}
 
 
 # ---------------------------------------------------------------- helpers

@@ -444,3 +444,40 @@ def test_residue_classes_c5_slice(sel):
         assert (g0["counts"] == g["counts"]).all() and (g0["cycles"] == g["cycles"]).all()
         assert (g0["decision"] == g["decision"]).all()
     assert g0["stats"]["wa_residue_classes"] > 0 and g16["stats"]["wa_residue_classes"] == 0
+
+
+def _distinct_problems(b):
+    """(nest, B class) pairs the batch's valid candidates refer to."""
+    B = b.launches["block"][b.cands["launch_id"]].astype(np.int64)
+    cls = np.where(B % 32 == 0, 32, B)
+    return len(set(zip(b.cands["nest_id"].tolist(), cls.tolist())))
+
+
+def test_direct_and_hashed_problem_ids_agree(sel):
+    """Direct problem ids (launch table <= 1024 entries) and the slot-table path
+    (forced by padding the launch table past 1024 entries) give identical
+    counts, cycles and decisions, and both count each distinct (nest, B class)
+    problem once -- including a slice where most direct ids are unused."""
+    b = gen.generate(5, 0, 3 * 768 * 7)
+    keep = np.nonzero((b.cands["launch_id"] % 3 != 1) & (np.arange(len(b)) % 5 != 0))[0]
+    b = b.select(keep)
+    pad = np.zeros(1100, gen.LAUNCH_DTYPE)
+    pad["block"], pad["grid_max"] = 96, 65535
+    b_hashed = gen.Batch(b.cands, b.nests, b.accesses, np.concatenate([b.launches, pad]), b.devices)
+    g_direct, g_hashed = run_gpu(sel, b), run_gpu(sel, b_hashed)
+    ref = oracle.evaluate(b)
+    assert_parity(g_direct, ref, ctx="direct ids")
+    assert_parity(g_hashed, ref, ctx="slot-table ids")
+    n = _distinct_problems(b)
+    assert g_direct["stats"]["n_problems"] == n == g_hashed["stats"]["n_problems"]
+
+
+def test_direct_ids_sparse_nests(sel):
+    """Many nests, few candidates each (nests x classes > candidates): the plan
+    falls back to the slot table; counts still exact."""
+    b = gen.generate(5, 0, 768 * 40)
+    idx = np.arange(0, len(b), 97)
+    b = b.select(idx)
+    g = run_gpu(sel, b)
+    assert_parity(g, oracle.evaluate(b), ctx="sparse")
+    assert g["stats"]["n_problems"] == _distinct_problems(b)

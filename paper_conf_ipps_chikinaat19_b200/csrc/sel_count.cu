@@ -1394,7 +1394,10 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
 #define SEL_LANE_MIN_BLOCKS 2
 #endif
 constexpr uint32_t kLaneGrp = 4;        // problems of a unit counted together
-constexpr uint32_t kLaneTile = 2048;    // units sorted per block tile
+#ifndef SEL_LANE_TILE
+#define SEL_LANE_TILE 1024
+#endif
+constexpr uint32_t kLaneTile = SEL_LANE_TILE;   // units sorted per block tile
 constexpr uint32_t kLaneKeyBits = 8;
 constexpr uint32_t kLaneKeys = 1u << kLaneKeyBits;
 constexpr size_t kLaneSmem = (size_t(kLaneRows) * kLaneThreads + kLaneTile + kLaneKeys) * sizeof(uint32_t);

@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
             continue;
         }
         if (!dedup) {
-            cand_pid[c] = uint32_t(c);
+            cand_pid[c] = st ? kNoProblem : uint32_t(c);          // kNoProblem <=> candidate invalid (all modes)
             prob_nest[c] = st ? kNoProblem : cd.nest_id;
             prob_B[c] = st ? 0u : t.launches[cd.launch_id].block;
             continue;

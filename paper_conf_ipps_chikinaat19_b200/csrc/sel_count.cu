@@ -1539,13 +1539,21 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                         const uint64_t q = u * ncls + g0 + c;
                         sW += uint64_t(WR[c]) * a.prob_cnt[q * kCntStride + 5];
                         sOps += z[c].ops;
-                        if (z[c].W) {
+                        {   // the only writer so far (k_problem_w leaves these counters unzeroed): store
                             unsigned long long* pc = a.prob_cnt + q * kCntStride;
-                            atomicAdd(pc + 0, (unsigned long long)z[c].W);
-                            atomicAdd(pc + 1, (unsigned long long)z[c].L);
-                            atomicAdd(pc + 2, (unsigned long long)z[c].S);
-                            atomicAdd(pc + 3, (unsigned long long)z[c].C);
-                            atomicAdd(pc + 4, (unsigned long long)z[c].U);
+                            if (a.hdr->n_parts == 1) {
+                                pc[0] = z[c].W;
+                                pc[1] = z[c].L;
+                                pc[2] = z[c].S;
+                                pc[3] = z[c].C;
+                                pc[4] = z[c].U;
+                            } else if (z[c].W) {
+                                atomicAdd(pc + 0, (unsigned long long)z[c].W);
+                                atomicAdd(pc + 1, (unsigned long long)z[c].L);
+                                atomicAdd(pc + 2, (unsigned long long)z[c].S);
+                                atomicAdd(pc + 3, (unsigned long long)z[c].C);
+                                atomicAdd(pc + 4, (unsigned long long)z[c].U);
+                            }
                         }
                     }
                 }

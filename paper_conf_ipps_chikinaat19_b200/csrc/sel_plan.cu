@@ -294,13 +294,20 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 }
 
 // closed-form W = WR * M_it per problem (+ nest validation V3-V6)
+// The counters of a small problem with W > 0 are not zeroed here: in a
+// single-part call the lane kernel thread that counts it STORES its sums
+// (k_queue adds the handed-over accesses afterwards).
 __device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
                                               const uint32_t* prob_B, unsigned long long* prob_W,
                                               unsigned long long* prob_WR, uint8_t* prob_status,
-                                              unsigned long long* prob_cnt, int lane_ok) {
-    for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
+                                              unsigned long long* prob_cnt, int lane_ok, bool one_part) {
     prob_status[q] = st;
-    if (st) { prob_W[q] = 0; prob_WR[q] = 0; prob_cnt[q * kCntStride + 5] = 0; return; }
+    if (st) {
+        for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
+        prob_W[q] = 0;
+        prob_WR[q] = 0;
+        return;
+    }
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
     prob_cnt[q * kCntStride + 5] = M_it;
@@ -308,6 +315,8 @@ __device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, 
     const uint64_t W = WR * M_it;
     const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
     prob_W[q] = small ? 0ull : W;
+    if (!(small && W != 0 && one_part))
+        for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
 }
 
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
@@ -404,7 +413,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                     const bool u = c < 32 ? ((um >> c) & 1u) : prob_nest[q] != kNoProblem;
                     used += u ? 1u : 0u;
                     problem_w_one(q, nest, u ? st : uint8_t(SEL_EINVAL), st == SEL_OK ? M_it : 0ull, prob_B, prob_W,
-                                  prob_WR, prob_status, prob_cnt, lane_ok);
+                                  prob_WR, prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
                 }
             }
             __syncwarp();
@@ -424,7 +433,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
             nest = t.nests[nid];
             st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
         }
-        problem_w_one(q, nest, st, M_it, prob_B, prob_W, prob_WR, prob_status, prob_cnt, lane_ok);
+        problem_w_one(q, nest, st, M_it, prob_B, prob_W, prob_WR, prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
     }
 }
 

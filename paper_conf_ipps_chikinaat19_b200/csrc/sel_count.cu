@@ -75,6 +75,7 @@ struct CountArgs {
     uint32_t closed_form;               // resolve warp-reps with uniform lane flags in closed form
     uint32_t residue_classes;           // whole arithmetic-lane warp-reps by residue classes (count_hist)
     unsigned long long* queue;          // small problems handed from k_lane_problems to k_queue
+    const uint8_t* nest_key;            // direct mode: shape key per nest (k_problem_w)
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -1390,6 +1391,9 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
 // warp's lanes run nests of one shape side by side instead of 32 different
 // loop structures.  A thread hands the accesses it cannot count to the warp
 // kernel (k_queue): entry = problem << 32 | mask of handed accesses.
+#ifndef SEL_LANE_NEST_KEY
+#define SEL_LANE_NEST_KEY 1
+#endif
 #ifndef SEL_LANE_MIN_BLOCKS
 #define SEL_LANE_MIN_BLOCKS 2
 #endif
@@ -1402,15 +1406,18 @@ constexpr uint32_t kLaneKeyBits = 8;
 constexpr uint32_t kLaneKeys = 1u << kLaneKeyBits;
 constexpr size_t kLaneSmem = (size_t(kLaneRows) * kLaneThreads + kLaneTile + kLaneKeys) * sizeof(uint32_t);
 
-// shape key of a unit: accesses, loop depth, collapse (keys that also hash the
-// first accesses' counting paths and element sizes cost more in descriptor loads
-// than they gained in SIMT efficiency: profiles/r01_variants_v8/)
+// shape key of a unit: direct mode, the nest's key from k_problem_w (one
+// coalesced byte; it also hashes the accesses' counting paths and element
+// sizes, which k_problem_w sees anyway -- loading descriptors here for that
+// cost more than it gained, profiles/r01_variants_v8/); otherwise accesses,
+// loop depth and collapse of the problem's nest.
 __device__ __forceinline__ uint32_t lane_unit_key(const CountArgs& a, uint64_t u, bool direct) {
+#if SEL_LANE_NEST_KEY
+    if (direct) return a.nest_key[u];
+#endif
     const uint32_t nid = direct ? uint32_t(u) : a.prob_nest[u];
     if (nid == kNoProblem) return 0u;
-    const sel_nest* np = a.nests + nid;
-    const uint32_t na = np->n_access < 31u ? np->n_access : 31u;
-    return (na << 3) | (uint32_t(np->depth & 3u) << 1) | (np->par_dims == 2 ? 1u : 0u);
+    return nest_shape_key(a.nests[nid]);
 }
 
 template <int MODE>
@@ -1782,7 +1789,7 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
                 (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u,
-                w.queue};
+                w.queue, w.nest_key};
     prof_before_count(s);
     if (mode == 0) launch_mode<0>(a, s);
     else if (mode == 1) launch_mode<1>(a, s);

@@ -41,7 +41,7 @@ static_assert(sizeof(WsHeader) == 256, "header size");
 
 struct WsLayout {
     size_t hdr, slots, nest_base, cand_pid, prob_nest, prob_B, prob_W, prob_WR, prob_cnt,
-        prob_status, cand_status, queue, prob_md, cls, scan_tmp, total;
+        prob_status, cand_status, queue, prob_md, cls, nest_key, scan_tmp, total;
 };
 
 __host__ __device__ inline size_t ws_align(size_t x) { return (x + 255) & ~size_t(255); }
@@ -70,6 +70,7 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
     L.queue = o;      o = ws_align(o + n * sizeof(uint64_t));
     L.prob_md = o;    o = ws_align(o + n * kProbModelBytes);
     L.cls = o;        o = ws_align(o + 2 * kClsMax * sizeof(uint32_t));
+    L.nest_key = o;   o = ws_align(o + n);
     uint64_t big = n > n_nests ? n : n_nests;
     L.scan_tmp = o;   o = ws_align(o + scan_blocks(big) * sizeof(uint64_t) * 2);
     L.total = o;
@@ -112,6 +113,24 @@ __device__ __forceinline__ uint8_t validate_candidate(const sel_candidate& c, co
     const sel_launch l = t.launches[c.launch_id];
     if (l.block < 1 || l.block > 1024 || l.grid_max < 1) return SEL_EINVAL;
     return SEL_OK;
+}
+
+// Shape key of a nest for the lane kernel's tile sort: accesses, loop depth,
+// collapse, how many accesses take each counting path (uniform / residue
+// classes depth <= 1 / depth 2 / warp kernel; 8-bit counts in `paths`) and
+// which element sizes occur (`emask`), hashed to 8 bits -- threads of a warp
+// then run nests whose loops and branches match.  A hint only: collisions mix
+// shapes, nothing else.
+__device__ __forceinline__ uint8_t nest_shape_key(const sel_nest& n, uint32_t paths, uint32_t emask) {
+    const uint32_t na = n.n_access < 31u ? n.n_access : 31u;
+    uint32_t h = (na << 3) | (uint32_t(n.depth & 3u) << 1) | (n.par_dims == 2 ? 1u : 0u);
+    h = h * 0x9E3779B1u + paths;
+    h = h * 0x9E3779B1u + emask;
+    return uint8_t((h * 0x9E3779B1u) >> 24);
+}
+__device__ __forceinline__ uint8_t nest_shape_key(const sel_nest& n) {
+    const uint32_t na = n.n_access < 31u ? n.n_access : 31u;
+    return uint8_t((na << 3) | (uint32_t(n.depth & 3u) << 1) | (n.par_dims == 2 ? 1u : 0u));
 }
 
 // Nest-level checks V3-V6, split so that the accesses can be checked by

@@ -24,6 +24,7 @@ struct WsPtrs {
     unsigned long long* queue;       // (problem << 32 | first WA) handed from the lane to the warp kernel
     void* prob_md;                   // per problem: ProbModel (sel_model.cu)
     uint32_t* cls;                   // [kClsMax] class index per launch, [kClsMax..) B class per index
+    uint8_t* nest_key;               // direct mode: shape key per nest (k_problem_w -> k_lane_problems)
     unsigned long long* scan_tmp;
 };
 

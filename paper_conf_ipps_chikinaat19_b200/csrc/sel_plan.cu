@@ -322,7 +322,7 @@ __device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, 
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
-                                                   unsigned long long* prob_cnt, int lane_ok) {
+                                                   unsigned long long* prob_cnt, int lane_ok, uint8_t* nest_key) {
     const uint64_t nq = hdr->n_problems;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     if (hdr->direct) {
@@ -334,6 +334,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
         // writes its n_cls problems.
         __shared__ uint32_t s_flags[8][32];
         __shared__ unsigned long long s_mit[8][32];
+        __shared__ uint32_t s_paths[8][32], s_emask[8][32];
         const uint32_t ncls = hdr->n_cls;
         const uint64_t nn = ncls ? nq / ncls : 0;
         const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -361,6 +362,8 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
             const uint32_t tot = __shfl_sync(kFull, incl, 31);
             const uint64_t P = smul(nest.P0, nest.P1);
             s_flags[wib][lane] = 0u;
+            s_paths[wib][lane] = 0u;
+            s_emask[wib][lane] = 0u;
             s_mit[wib][lane] = 0ull;
             __syncwarp();
             for (uint32_t j0 = 0; j0 < tot; j0 += 32) {
@@ -382,9 +385,18 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                 const uint64_t T[3] = {eff_trip(__shfl_sync(kFull, nest.trip[0], own)),
                                        eff_trip(__shfl_sync(kFull, nest.trip[1], own)),
                                        eff_trip(__shfl_sync(kFull, nest.trip[2], own))};
-                uint32_t fl = 0;
+                uint32_t fl = 0, paths = 0, em = 0;
                 uint64_t Mk = 0;
-                if (j < tot) fl = access_check(t.accesses[aoff + (j - ex)], pd, dp, Po, P0o, P1o, T, &Mk);
+                if (j < tot) {
+                    const sel_access ac = t.accesses[aoff + (j - ex)];
+                    fl = access_check(ac, pd, dp, Po, P0o, P1o, T, &Mk);
+                    // the counting path the lane kernel will take (for its shape sort), 8-bit counts
+                    const uint64_t g = uabs(ac.c_par[0]);
+                    const uint32_t path = (g == 0 || g >= 128) ? 0u : ac.elem_bytes < 4 ? 3u : ac.depth <= 1 ? 1u :
+                                          ac.depth == 2 ? 2u : 3u;
+                    paths = 1u << (8u * path);
+                    em = 1u << (__ffs(ac.elem_bytes) & 31);
+                }
                 // segmented (by owner) saturating sum over the lanes of this round
                 const bool in = j < tot;
 #pragma unroll
@@ -392,9 +404,12 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                     const uint64_t y = __shfl_up_sync(kFull, Mk, o);
                     const uint32_t yf = __shfl_up_sync(kFull, fl, o);
                     const int yo = __shfl_up_sync(kFull, own, o);
+                    const uint32_t yp = __shfl_up_sync(kFull, paths, o), ye = __shfl_up_sync(kFull, em, o);
                     if (lane >= o && yo == own) {
                         Mk = sadd(Mk, y);
                         fl |= yf;
+                        paths += yp;
+                        em |= ye;
                     }
                 }
                 const int nxt = __shfl_down_sync(kFull, own, 1);
@@ -402,10 +417,13 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                 if (tail) {                                     // one lane per owner per round
                     s_mit[wib][own] = sadd(s_mit[wib][own], Mk);
                     s_flags[wib][own] |= fl;
+                    s_paths[wib][own] += paths;
+                    s_emask[wib][own] |= em;
                 }
                 __syncwarp();
             }
             if (i < nn) {
+                nest_key[i] = nest_shape_key(nest, s_paths[wib][lane], s_emask[wib][lane]);
                 const uint64_t M_it = s_mit[wib][lane];
                 const uint8_t st = nest_status(pre, s_flags[wib][lane], P, M_it);
                 for (uint32_t c = 0; c < ncls; c++) {
@@ -487,7 +505,8 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
     k_problem_w<<<gb, 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
                                                           w.prob_status, w.prob_cnt,
                                                           (flags & (SEL_F_MATCH_ANY | SEL_F_EXPAND_ALL |
-                                                                    SEL_F_WARP_PROBLEMS)) ? 0 : 1);
+                                                                    SEL_F_WARP_PROBLEMS)) ? 0 : 1,
+                                                          w.nest_key);
     note_launch(2);
     if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s)) != cudaSuccess) return e;
     k_plan_stats<<<1, 1, 0, s>>>(w.hdr, w.prob_W);

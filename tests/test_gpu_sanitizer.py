@@ -1,6 +1,8 @@
 """compute-sanitizer over the CUDA path on small configs:
 memcheck (out-of-bounds / misaligned accesses), racecheck (shared-memory
-hazards in the scan kernels) and synccheck (barrier / warp-sync misuse),
+hazards in the scan, sort and histogram kernels) and synccheck (barrier /
+warp-sync misuse) on c1-c3 samples, a c5 slice and hand-written shapes that
+reach every counting kernel (lane, queue with cp.async prefetch, big),
 each expected to report zero errors."""
 import os
 import shutil
@@ -19,8 +21,24 @@ import sys, numpy as np, torch
 sys.path.insert(0, %r)
 import gen
 import paper_conf_ipps_chikinaat19_b200 as sel
-for cfg, idx, flags in ((1, None, 0), (1, None, 2), (3, np.arange(0, 3000, 7), 0), (2, np.arange(0, 108, 9), 1)):
-    b = gen.generate(cfg) if idx is None else gen.generate(cfg).select(idx)
+# queue-kernel and lane-kernel shapes: element sizes 1/2 (handed to the warp kernel), depth 3,
+# blocks that 32 does not divide (warp-rep classes), depth-2 residue histograms
+launches = np.zeros(3, gen.LAUNCH_DTYPE)
+launches[0], launches[1], launches[2] = (48, 65535, 0, 0), (200, 3, 0, 0), (128, 65535, 0, 0)
+items = []
+for e, d, cp in ((1, 1, 3), (2, 3, 6), (4, 2, 4), (8, 1, -8), (16, 2, 16), (4, 1, 100)):
+    a = gen.make_access(base=(1 << 30) + 7 * e, c_par=(cp,), c_inner=[e * 3, 96 * e, 5 * e][:d], elem_bytes=e, depth=d)
+    for li in range(3):
+        items.append(dict(P0=97 + 11 * li, trip=[9, 5, 3][:d], depth=d, comp=[1.0] * (d + 1), accesses=[a, a], launch=li))
+custom = gen.custom_batch(items, launches_=launches)
+for cfg, idx, flags in ((1, None, 0), (1, None, 2), (3, np.arange(0, 3000, 7), 0), (2, np.arange(0, 108, 9), 1),
+                        (5, None, 0), ("custom", None, 0), ("custom", None, 8)):
+    if cfg == "custom":
+        b = custom
+    elif cfg == 5:
+        b = gen.generate(5, 0, 768 * 3)
+    else:
+        b = gen.generate(cfg) if idx is None else gen.generate(cfg).select(idx)
     ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b), flags)
     c = sel._as_bytes_tensor(b.cands, "candidate")
     r = ev.evaluate(c, want_counts=True, want_t_gpu=True)

@@ -1397,7 +1397,10 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
 #ifndef SEL_LANE_MIN_BLOCKS
 #define SEL_LANE_MIN_BLOCKS 2
 #endif
-constexpr uint32_t kLaneGrp = 4;        // problems of a unit counted together
+#ifndef SEL_LANE_GRP
+#define SEL_LANE_GRP 3
+#endif
+constexpr uint32_t kLaneGrp = SEL_LANE_GRP;   // problems of a unit counted together
 #ifndef SEL_LANE_TILE
 #define SEL_LANE_TILE 1024
 #endif

@@ -1402,7 +1402,7 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
 #endif
 constexpr uint32_t kLaneGrp = SEL_LANE_GRP;   // problems of a unit counted together
 #ifndef SEL_LANE_TILE
-#define SEL_LANE_TILE 1024
+#define SEL_LANE_TILE 4096
 #endif
 constexpr uint32_t kLaneTile = SEL_LANE_TILE;   // units sorted per block tile
 constexpr uint32_t kLaneKeyBits = 8;

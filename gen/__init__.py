@@ -23,6 +23,7 @@ DEVICE_DTYPE = np.dtype([
     ("sm_clock_hz", "<f8"), ("mem_bw_Bps", "<f8"), ("link_bw_Bps", "<f8"),
     ("launch_overhead_s", "<f8"), ("mem_ld_cycles", "<f8"), ("dep_del_coal", "<f8"),
     ("dep_del_uncoal", "<f8"), ("issue_cycles", "<f8"),
+    ("reg_alloc_unit", "<i4"), ("warp_alloc_gran", "<i4"), ("smem_alloc_unit", "<i4"), ("txn_sectors", "<i4"),
 ])
 ACCESS_DTYPE = np.dtype([
     ("base", "<i8"), ("c_par", "<i8", (2,)), ("c_inner", "<i8", (3,)),

@@ -166,16 +166,21 @@ const char* selgen_shape_name(int s) { return (s >= 0 && s < 24) ? SHAPES[s].nam
 /* ------------------------------------------------------- device / launch */
 int selgen_device_sets(gen_device_params* o) {
     /* Table III names the parameters but its values were lost;
-     * these are builder-chosen public/vendor figures (R23). */
+     * these are builder-chosen public/vendor figures (R23).  The
+     * last four fields are NEXT row f4's (F4c, F4d): register
+     * allocation unit 256 registers per warp, warp allocation granularity 4,
+     * shared-memory allocation unit 256 B (the CUDA occupancy calculator's
+     * values for these generations), and the transaction unit -- 128 B lines
+     * (H&K) for K80 / P100 / V100 as in the paper, 32 B sectors for B200. */
     const gen_device_params d[4] = {
         /* K80, one GK210 */
-        {13, 64, 2048, 16, 131072, 114688, 0.875e9, 240.48e9, 12.0e9, 5.0e-6, 440.0, 4.0, 12.0, 4.0},
+        {13, 64, 2048, 16, 131072, 114688, 0.875e9, 240.48e9, 12.0e9, 5.0e-6, 440.0, 4.0, 12.0, 4.0, 256, 4, 256, 0},
         /* P100 SXM2 */
-        {56, 64, 2048, 32, 65536, 65536, 1.480e9, 732.0e9, 32.0e9, 4.0e-6, 500.0, 4.0, 10.0, 2.0},
+        {56, 64, 2048, 32, 65536, 65536, 1.480e9, 732.0e9, 32.0e9, 4.0e-6, 500.0, 4.0, 10.0, 2.0, 256, 4, 256, 0},
         /* V100 SXM2 (AC922, NVLink 2: 3 bricks x 25 GB/s) */
-        {80, 64, 2048, 32, 65536, 98304, 1.530e9, 900.0e9, 75.0e9, 4.0e-6, 440.0, 4.0, 10.0, 2.0},
+        {80, 64, 2048, 32, 65536, 98304, 1.530e9, 900.0e9, 75.0e9, 4.0e-6, 440.0, 4.0, 10.0, 2.0, 256, 4, 256, 0},
         /* B200 */
-        {148, 64, 2048, 32, 65536, 233472, 1.965e9, 7.7e12, 55.0e9, 3.0e-6, 600.0, 4.0, 8.0, 2.0},
+        {148, 64, 2048, 32, 65536, 233472, 1.965e9, 7.7e12, 55.0e9, 3.0e-6, 600.0, 4.0, 8.0, 2.0, 256, 4, 256, 1},
     };
     memcpy(o, d, sizeof d);
     return 4;

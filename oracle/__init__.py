@@ -14,7 +14,9 @@ import subprocess
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+# SEL_ORACLE_LIB: load a prebuilt variant instead (scripts/mutate_oracle.py runs
+# the pins against deliberately broken copies of oracle.c)
+_LIB_PATH = os.environ.get("SEL_ORACLE_LIB") or os.path.join(_HERE, "liboracle.so")
 
 RESULT_DTYPE = np.dtype([
     ("W", "<u8"), ("L", "<u8"), ("S", "<u8"), ("C", "<u8"), ("U", "<u8"), ("WR", "<u8"),
@@ -36,6 +38,8 @@ _lib = None
 def build(force: bool = False) -> str:
     src = os.path.join(_HERE, "oracle.c")
     hdr = os.path.join(_HERE, "oracle.h")
+    if os.environ.get("SEL_ORACLE_LIB"):
+        return _LIB_PATH
     if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < max(
             os.path.getmtime(src), os.path.getmtime(hdr)):
         # -ffp-contract=off: no FMA contraction, so the fp64 model sequence

@@ -20,11 +20,15 @@
  * Readings R1-R31 resolve what the paper leaves open.
  *
  * Parity pins: tests/test_oracle_*.py (closed forms, brute force in pure
- * Python, the paper's worked examples, invariants).  The Hong & Kim
- * equations that PAPER.md does not print (Mem_L, Departure_delay,
- * MWP_Without_BW, #Rep, Comp/Mem cycles; readings R2, R5) are
- * "parity unpinned" against the paper: only their special cases and
- * invariants are checked.
+ * Python, the paper's worked examples, invariants) and, for the model half,
+ * tests/test_oracle_hand.py: hand-computed candidates for every case of
+ * Fig. 4, the bandwidth branch of Fig. 5, mixed coalesced / uncoalesced
+ * weights, a non-integer #Rep, #OMP_Rep, an exact T_gpu and the NEXT row f4
+ * extensions; scripts/mutate_oracle.py shows that 29 single-term mutations
+ * of this file each fail one of them.  What stays unverifiable from PAPER.md
+ * is the FORM of the Hong & Kim equations it does not print (Mem_L,
+ * Departure_delay, MWP_Without_BW, #Rep, Comp/Mem cycles; readings R2, R5):
+ * the pins fix this code to those equations as DESIGN.md restates them.
  */
 #include "oracle.h"
 #include <math.h>
@@ -97,7 +101,8 @@ static int valid_device(const or_device* d) {
            d->max_blocks_per_sm >= 1 && d->regs_per_sm >= 0 && d->smem_per_sm >= 0 &&
            d->sm_clock_hz > 0 && d->mem_bw_Bps > 0 && d->link_bw_Bps > 0 &&
            d->launch_overhead_s >= 0 && d->mem_ld_cycles > 0 && d->dep_del_coal > 0 &&
-           d->dep_del_uncoal > 0 && d->issue_cycles > 0;
+           d->dep_del_uncoal > 0 && d->issue_cycles > 0 && d->reg_alloc_unit >= 0 && d->warp_alloc_gran >= 0 &&
+           d->smem_alloc_unit >= 0 && (d->txn_sectors == 0 || d->txn_sectors == 1);
 }
 
 /* ------------------------------------------------------------------ model */
@@ -132,10 +137,27 @@ void oracle_model(const or_device* dev, const or_nest* nest, const or_access* ac
     uint64_t abps = (uint64_t)dev->max_blocks_per_sm;
     abps = umin(abps, (uint64_t)dev->max_warps_per_sm / r->wpb);
     abps = umin(abps, (uint64_t)dev->max_threads_per_sm / B);
-    if (launch->regs_per_thread > 0)
-        abps = umin(abps, (uint64_t)dev->regs_per_sm / ((uint64_t)launch->regs_per_thread * B));
-    if (launch->smem_per_block > 0)
-        abps = umin(abps, (uint64_t)dev->smem_per_sm / (uint64_t)launch->smem_per_block);
+    if (launch->regs_per_thread > 0) {
+        if (dev->reg_alloc_unit > 0) {
+            /* NEXT row f4, allocation granularity (reading F4c): registers are
+             * allocated per warp in units of reg_alloc_unit, and the warps the
+             * register file holds are rounded down to warp_alloc_gran */
+            const uint64_t unit = (uint64_t)dev->reg_alloc_unit;
+            const uint64_t regs_per_warp = ceil_div((uint64_t)launch->regs_per_thread * 32, unit) * unit;
+            uint64_t warps = (uint64_t)dev->regs_per_sm / regs_per_warp;
+            if (dev->warp_alloc_gran > 1) warps = (warps / (uint64_t)dev->warp_alloc_gran) * (uint64_t)dev->warp_alloc_gran;
+            abps = umin(abps, warps / r->wpb);
+        } else {
+            abps = umin(abps, (uint64_t)dev->regs_per_sm / ((uint64_t)launch->regs_per_thread * B));
+        }
+    }
+    if (launch->smem_per_block > 0) {
+        /* F4c: shared memory is allocated per block in units of smem_alloc_unit */
+        uint64_t smem_b = (uint64_t)launch->smem_per_block;
+        if (dev->smem_alloc_unit > 0)
+            smem_b = ceil_div(smem_b, (uint64_t)dev->smem_alloc_unit) * (uint64_t)dev->smem_alloc_unit;
+        abps = umin(abps, (uint64_t)dev->smem_per_sm / smem_b);
+    }
     abps = umin(abps, ceil_div(r->G, (uint64_t)dev->num_sms));
     r->abps = abps;
     r->active_sms = umin(r->G, (uint64_t)dev->num_sms);
@@ -156,7 +178,13 @@ void oracle_model(const or_device* dev, const or_nest* nest, const or_access* ac
         r->hk_case = 0;
         Exec = (((issue * comp) * N) * Rep) * (double)r->R;
     } else {
-        const uint64_t W = r->W, C = r->C, U = r->U, S = r->S, WR = r->WR;
+        const uint64_t W = r->W, S = r->S, WR = r->WR;
+        /* NEXT row f4, 32 B-sector transactions (reading F4d): every
+         * warp-access is one class whose memory transactions are its distinct
+         * sectors -- H&K's inputs with #Coal = 0 and uncoalesced transactions
+         * U = S.  Otherwise 128 B lines with the R11 classes. */
+        const uint64_t C = dev->txn_sectors ? 0 : r->C;
+        const uint64_t U = dev->txn_sectors ? S : r->U;
         const double n_coal = (double)C / (double)WR;            /* #Coal_Mem_insts per warp */
         const double n_unc = (double)(W - C) / (double)WR;       /* #Uncoal_Mem_insts per warp */
         const double mem = (double)r->M_it;                      /* #Mem_insts (R4, R14) */
@@ -396,7 +424,9 @@ size_t oracle_offsetof(int which, int field) {
         OFF(or_device, max_threads_per_sm), OFF(or_device, max_blocks_per_sm), OFF(or_device, regs_per_sm),
         OFF(or_device, smem_per_sm), OFF(or_device, sm_clock_hz), OFF(or_device, mem_bw_Bps),
         OFF(or_device, link_bw_Bps), OFF(or_device, launch_overhead_s), OFF(or_device, mem_ld_cycles),
-        OFF(or_device, dep_del_coal), OFF(or_device, dep_del_uncoal), OFF(or_device, issue_cycles)};
+        OFF(or_device, dep_del_coal), OFF(or_device, dep_del_uncoal), OFF(or_device, issue_cycles),
+        OFF(or_device, reg_alloc_unit), OFF(or_device, warp_alloc_gran), OFF(or_device, smem_alloc_unit),
+        OFF(or_device, txn_sectors)};
     static const size_t acc[] = {OFF(or_access, base), OFF(or_access, c_par), OFF(or_access, c_inner),
         OFF(or_access, elem_bytes), OFF(or_access, depth), OFF(or_access, is_store)};
     static const size_t nest[] = {OFF(or_nest, P0), OFF(or_nest, P1), OFF(or_nest, trip), OFF(or_nest, par_dims),

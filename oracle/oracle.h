@@ -20,6 +20,8 @@ typedef struct {
     int32_t num_sms, max_warps_per_sm, max_threads_per_sm, max_blocks_per_sm, regs_per_sm, smem_per_sm;
     double sm_clock_hz, mem_bw_Bps, link_bw_Bps, launch_overhead_s,
            mem_ld_cycles, dep_del_coal, dep_del_uncoal, issue_cycles;
+    /* NEXT row f4: allocation granularity (F4c) and the transaction unit (F4d) */
+    int32_t reg_alloc_unit, warp_alloc_gran, smem_alloc_unit, txn_sectors;
 } or_device;
 
 typedef struct {

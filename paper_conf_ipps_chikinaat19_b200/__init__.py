@@ -71,7 +71,7 @@ def load_device_params(sets) -> None:
     """sel_load_device_params: copy 1..16 device parameter sets (host)."""
     a = np.ascontiguousarray(sets)
     if a.dtype.itemsize != _REC_SIZE["device"]:
-        raise ValueError("device parameter records must be 88 bytes")
+        raise ValueError(f"device parameter records must be {_REC_SIZE['device']} bytes")
     _lib.check(_lib.lib().sel_load_device_params(a.ctypes.data, len(a)))
 
 

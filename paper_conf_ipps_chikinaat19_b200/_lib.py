@@ -37,7 +37,9 @@ class DeviceParams(ctypes.Structure):
                 ("sm_clock_hz", ctypes.c_double), ("mem_bw_Bps", ctypes.c_double),
                 ("link_bw_Bps", ctypes.c_double), ("launch_overhead_s", ctypes.c_double),
                 ("mem_ld_cycles", ctypes.c_double), ("dep_del_coal", ctypes.c_double),
-                ("dep_del_uncoal", ctypes.c_double), ("issue_cycles", ctypes.c_double)]
+                ("dep_del_uncoal", ctypes.c_double), ("issue_cycles", ctypes.c_double),
+                ("reg_alloc_unit", ctypes.c_int32), ("warp_alloc_gran", ctypes.c_int32),
+                ("smem_alloc_unit", ctypes.c_int32), ("txn_sectors", ctypes.c_int32)]
 
 
 class Access(ctypes.Structure):

@@ -131,7 +131,9 @@ int sel_load_device_params(const sel_device_params* h, int n_sets) {
         const bool ok = d.num_sms >= 1 && d.max_warps_per_sm >= 1 && d.max_threads_per_sm >= 1 &&
                         d.max_blocks_per_sm >= 1 && d.regs_per_sm >= 0 && d.smem_per_sm >= 0 &&
                         d.sm_clock_hz > 0 && d.mem_bw_Bps > 0 && d.link_bw_Bps > 0 && d.launch_overhead_s >= 0 &&
-                        d.mem_ld_cycles > 0 && d.dep_del_coal > 0 && d.dep_del_uncoal > 0 && d.issue_cycles > 0;
+                        d.mem_ld_cycles > 0 && d.dep_del_coal > 0 && d.dep_del_uncoal > 0 && d.issue_cycles > 0 &&
+                        d.reg_alloc_unit >= 0 && d.warp_alloc_gran >= 0 && d.smem_alloc_unit >= 0 &&
+                        (d.txn_sectors == 0 || d.txn_sectors == 1);
         if (!ok) return fail(SEL_EINVAL, "invalid device parameter set%s");
     }
     int ndev = 0;
@@ -310,7 +312,9 @@ size_t sel_offsetof(int which, int field) {
         OFF(sel_device_params, mem_bw_Bps), OFF(sel_device_params, link_bw_Bps),
         OFF(sel_device_params, launch_overhead_s), OFF(sel_device_params, mem_ld_cycles),
         OFF(sel_device_params, dep_del_coal), OFF(sel_device_params, dep_del_uncoal),
-        OFF(sel_device_params, issue_cycles)};
+        OFF(sel_device_params, issue_cycles), OFF(sel_device_params, reg_alloc_unit),
+        OFF(sel_device_params, warp_alloc_gran), OFF(sel_device_params, smem_alloc_unit),
+        OFF(sel_device_params, txn_sectors)};
     static const size_t acc[] = {OFF(sel_access, base), OFF(sel_access, c_par), OFF(sel_access, c_inner),
         OFF(sel_access, elem_bytes), OFF(sel_access, depth), OFF(sel_access, is_store)};
     static const size_t nest[] = {OFF(sel_nest, P0), OFF(sel_nest, P1), OFF(sel_nest, trip), OFF(sel_nest, par_dims),
@@ -338,7 +342,7 @@ size_t sel_offsetof(int which, int field) {
 
 }  // extern "C"
 
-static_assert(sizeof(sel_device_params) == 88, "sel_device_params layout");
+static_assert(sizeof(sel_device_params) == 104, "sel_device_params layout");
 static_assert(sizeof(sel_access) == 64, "sel_access layout");
 static_assert(sizeof(sel_nest) == 88, "sel_nest layout");
 static_assert(sizeof(sel_launch) == 16, "sel_launch layout");

@@ -172,7 +172,7 @@ def measured_peaks():
 
 NCU_REGION_KERNELS = {
     "plan": ("k_classes", "k_insert", "k_rank_slots", "k_scan_reduce", "k_scan_partials", "k_scan_down", "k_assign",
-             "k_finalize_plan", "k_problem_w", "k_plan_stats"),
+             "k_finalize_plan", "k_problem_w", "k_mark_big", "k_drop_unused", "k_plan_stats"),
     "count": ("k_lane_problems", "k_queue", "k_count"),
     "model": ("k_problem_model", "k_model_fused"),
 }
@@ -200,9 +200,10 @@ def ncu_region(ncu, region):
     return {"source": ncu.get("source"), "kernels": ks} if ks else {}
 
 
-def cpu_oracle_sample(batch, seconds: float, total_candidates: int):
+def cpu_oracle_sample(batch, seconds: float, total_candidates: int, keep=None):
     """The oracle (as it stands) on a bounded, deterministic sample of the
-    workload, on all host cores."""
+    workload, on all host cores.  ``keep`` (a dict) receives the sample's
+    indices and oracle records for the per-run parity check."""
     import oracle
     cores = os.cpu_count() or 1
     n = len(batch)
@@ -217,6 +218,8 @@ def cpu_oracle_sample(batch, seconds: float, total_candidates: int):
     t0 = time.perf_counter()
     r = oracle.evaluate(sub, threads=cores)
     dt = time.perf_counter() - t0
+    if keep is not None:
+        keep["idx"], keep["ref"] = idx, r
     return {"value": m / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
             "sample": f"{m} candidates evenly spaced over the {total_candidates}-candidate sweep "
                       f"({int(r['W'].sum())} warp-accesses, {dt:.1f} s)",
@@ -260,7 +263,7 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64+f64",
             "data": "synthetic", "config": {"workload": WORKLOAD, "candidates": total},
-            "wa_analysed_per_s": was / T,
+            "wa_expanded_per_s": was / T,
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                              "sample": f"each step {per_step} candidates strided over the {total}-candidate sweep"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -290,17 +293,22 @@ def run_ours(args):
     cands_host = torch.from_numpy(batch.cands.view(np.uint8).reshape(-1)).pin_memory()
     cands = cands_host.to(dev)
     stream = torch.cuda.current_stream(dev)
-    out = None
-    gathered = torch.empty(D.padded_len(total, world) * world, dtype=torch.uint8, device=dev) if world > 1 else None
+    # outputs preallocated once; with N > 1 the decisions land directly in this rank's slot of the
+    # all-gather buffer (D.DecisionGather: one in-place all_gather_into_tensor per step, no copies)
+    gatherer = D.DecisionGather(total, world, rank, dev) if world > 1 and not split else None
+    n_loc = len(batch)
+    out = {"decision": gatherer.slot if gatherer else torch.empty(n_loc, dtype=torch.uint8, device=dev),
+           "cycles": torch.empty(n_loc, dtype=torch.float64, device=dev),
+           "status": torch.empty(n_loc, dtype=torch.uint8, device=dev)}
 
     def step():
         nonlocal out
         if split:
             out = D.evaluate_split(cands, ev.tables, ev.workspace, rank, world, args.flags)
         else:
-            out = ev.evaluate(cands, out=out)
-            if world > 1:
-                D.gather_decisions(out["decision"], total, world, out=gathered)
+            ev.evaluate(cands, out=out)
+            if gatherer:
+                gatherer.gather()
 
     int_peak = {"alu": sel.int_peak(0), "fma": sel.int_peak(1), "both": sel.int_peak(2)}
     for _ in range(args.warmup):
@@ -308,7 +316,9 @@ def run_ours(args):
     torch.cuda.synchronize(dev)
     stats = ev.stats()
     sel.profile_enable(True)
-    for r in (sel.PROF_PLAN, sel.PROF_COUNT, sel.PROF_MODEL):
+    PROF = {"plan": sel.PROF_PLAN, "count": sel.PROF_COUNT, "model": sel.PROF_MODEL,
+            "k_model_fused": sel.PROF_K_MODEL, "k_lane_problems": sel.PROF_K_LANE, "k_problem_w": sel.PROF_K_PROBLEM_W}
+    for r in PROF.values():
         sel.profile_read_region(r)
     launches0 = sel.kernel_launches()
     D.barrier(world)
@@ -323,15 +333,14 @@ def run_ours(args):
     D.barrier(world)
     ms_local = e0.elapsed_time(e1)
     launches = sel.kernel_launches() - launches0
-    plan_ms, plan_launches = sel.profile_read_region(sel.PROF_PLAN)
-    count_ms, count_launches = sel.profile_read_region(sel.PROF_COUNT)
-    model_ms, model_launches = sel.profile_read_region(sel.PROF_MODEL)
+    prof = {k: sel.profile_read_region(r) for k, r in PROF.items()}       # name -> (ms, launches)
     sel.profile_enable(False)
     ms = D.max_over_ranks(ms_local, world, dev)
-    wa_analysed = D.sum_over_ranks(stats["wa_analysed"], world, dev)
+    wa_resolved = D.sum_over_ranks(stats["wa_resolved"], world, dev)
     wa_covered = D.sum_over_ranks(stats["wa_covered"], world, dev)
     n_invalid = D.sum_over_ranks(stats["n_invalid"], world, dev)
     wa_closed = D.sum_over_ranks(stats["wa_closed_form"], world, dev)
+    wa_expanded = D.sum_over_ranks(stats["wa_expanded"], world, dev)
     t_step = ms / 1e3 / args.steps
     clocks = clk.summary()
 
@@ -344,7 +353,6 @@ def run_ours(args):
         nests_h = torch.from_numpy(batch.nests.view(np.uint8).reshape(-1)).pin_memory()
         acc_h = torch.from_numpy(batch.accesses.view(np.uint8).reshape(-1)).pin_memory()
         h2d, d2h = sel.HostPipeline.bytes_per_step(cands_host, nests_h, acc_h, len(batch))
-        out = None                                     # free the device-resident outputs
         pipe = sel.HostPipeline(ev, cands_host, nests_h, acc_h)
         for k in range(max(1, args.warmup)):
             pipe.step(k, cands_host, nests_h, acc_h)
@@ -370,18 +378,18 @@ def run_ours(args):
     f_mhz = clocks["sm_mhz"] or measured_peaks().get("clocks_under_load", {}).get("sm_mhz_median", 1965.0)
     hbm_peak = measured_peaks().get("hbm_gbs")
     ncu = ncu_kernels()
-    per_launch = {"plan": plan_ms / max(plan_launches, 1), "count": count_ms / max(count_launches, 1),
-                  "model": model_ms / max(model_launches, 1)}
+    per_launch = {k: ms / max(k_n, 1) for k, (ms, k_n) in prof.items()}
     # counting kernels: INT bound.  peak = measured INT32 lane-op rate with the ALU and FMA pipes both
     # issuing (sel_int_peak mode 2), all SMs.  achieved = the nominal algorithmic lane-ops of the paths
     # the counting kernels took (sel_stats.alg_lane_ops) / their measured time
     peak_ops = int_peak["both"]
     wa_arith, wa_res, wa_cf = stats["wa_arith_lanes"], stats["wa_residue_classes"], stats["wa_closed_form"]
-    wa_lane = stats["wa_analysed"] - wa_cf - wa_arith - wa_res
+    wa_lane = stats["wa_resolved"] - wa_cf - wa_arith - wa_res
     avg_count_ms = per_launch["count"]
     achieved = stats["alg_lane_ops"] / (avg_count_ms / 1e3)
-    survey_eq = stats["wa_analysed"] * OPS_PER_WA / (avg_count_ms / 1e3)
-    roof_count = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
+    survey_eq = stats["wa_resolved"] * OPS_PER_WA / (avg_count_ms / 1e3)
+    roof_count = {"bound": "alu", "builder_weighted": True, "achieved": achieved / 1e12, "peak": peak_ops / 1e12,
+                  "unit": "Tops/s",
                   "frac": achieved / peak_ops, "traffic": ncu_region_traffic(ncu, "count"),
                   "kernel": "counting kernels (k_lane_problems + k_queue + k_count)",
                   "ms_per_launch": avg_count_ms, "share_of_step": avg_count_ms / (t_step * 1e3),
@@ -397,8 +405,9 @@ def run_ours(args):
                                         "note": "SURVEY §8(d)'s 224 lane-ops x every analysed warp-access / "
                                                 "counting time: the brute-force expansion rate the exact closed "
                                                 "forms stand in for (> 1 = faster than expanding at the INT peak)"},
-                  "note": ("achieved = nominal algorithmic lane-ops of the paths the counting kernels took "
-                           "(sel_stats.alg_lane_ops) / their time"),
+                  "note": ("NOT a measured counter: achieved = builder-weighted nominal lane-ops of the paths the "
+                           "counting kernels took (sel_stats.alg_lane_ops) / their time; the measured INT-pipe "
+                           "utilisation is int_pipe_ncu"),
                   "ncu": ncu_region(ncu, "count")}
     # model kernels (k_problem_model + k_model_fused): per candidate the 24 B record in, decision (1) +
     # cycles (8) + status (1) out -- HBM is the roofline of a streaming per-candidate kernel
@@ -419,8 +428,35 @@ def run_ours(args):
                          f"{PLAN_BYTES} B per candidate (record in, problem id + status out) + every nest (88 B) "
                          f"and access (64 B) record once")
     regions = {"plan": roof_plan, "count": roof_count, "model": roof_model}
-    dominant = max(per_launch, key=per_launch.get)
-    roofline = dict(regions[dominant], region=dominant)
+    # the dominant KERNEL (CUDA events around it alone, on the launching stream): k_model_fused against
+    # HBM on its algorithmic 34 B per candidate, or k_lane_problems / k_problem_w, whichever is longest
+    kern = {k: per_launch[k] for k in ("k_model_fused", "k_lane_problems", "k_problem_w")}
+    dominant = max(kern, key=kern.get)
+    kbytes = {"k_model_fused": (MODEL_BYTES * len(batch),
+                                f"{MODEL_BYTES} B per candidate (24 B record in; decision, cycles, status out)"),
+              "k_problem_w": (88 * n_nests + 64 * n_acc + 34 * len(batch) // 10,
+                              "every nest (88 B) and access (64 B) in, ~34 B per problem out"),
+              "k_lane_problems": (88 * n_nests + 64 * n_acc + 40 * (len(batch) * 3 // 32),
+                                  "every nest (88 B) and access (64 B) in, 40 B of counts per problem out")}
+    kb, kdesc = kbytes[dominant]
+    kms = kern[dominant]
+    ka = kb / (kms / 1e3) / 1e9
+    knc = ncu.get("kernels", {}).get(dominant, {})
+    roofline = {"bound": "hbm", "achieved": ka, "peak": hbm_peak, "unit": "GB/s",
+                "frac": ka / hbm_peak if hbm_peak else None,
+                "traffic": knc.get("dram_bytes"), "kernel": dominant, "ms_per_launch": kms,
+                "share_of_step": kms / (t_step * 1e3), "algorithmic_bytes_per_launch": kb, "bytes": kdesc,
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth, burst)",
+                "traffic_source": ncu.get("source"),
+                "ncu": {k: knc.get(k) for k in ("issue_active_pct", "warps_active_pct", "warp_instructions",
+                                                "fp64_cycles_pct", "alu_cycles_pct", "fma_cycles_pct")}}
+    # the north star's INT-pipe criterion: ncu sm__pipe_alu/fma_cycles_active of the counting kernel
+    lane_nc = ncu.get("kernels", {}).get("k_lane_problems", {})
+    int_pipe = {"kernel": "k_lane_problems", "source": ncu.get("source"),
+                "alu_cycles_pct": lane_nc.get("alu_cycles_pct"), "fma_cycles_pct": lane_nc.get("fma_cycles_pct"),
+                "alu_inst_pct": lane_nc.get("alu_pipe_pct"), "fma_inst_pct": lane_nc.get("fma_pipe_pct"),
+                "issue_active_pct": lane_nc.get("issue_active_pct"),
+                "ms_per_launch": per_launch["k_lane_problems"]}
     # the whole step against HBM: per candidate the 24 B record in, decision + cycles out
     step_hbm = {"bound": "hbm", "bytes_per_candidate": CAND_BYTES,
                 "achieved": CAND_BYTES * total / t_step / 1e9, "peak": hbm_peak, "unit": "GB/s"}
@@ -442,21 +478,60 @@ def run_ours(args):
                        "l2": (f"inputs larger than L2 ({24 * total / 1e9:.1f} GB of candidates per pass)"
                               if 24 * total > 126e6 else "inputs fit in L2 (not the metric workload)"),
                        "parallelism": parallelism},
-            "wa_analysed_per_s": wa_analysed / t_step, "wa_covered_per_s": wa_covered / t_step,
-            "wa_analysed_per_step": wa_analysed, "wa_covered_per_step": wa_covered, "invalid": n_invalid,
+            "wa_resolved_per_s": wa_resolved / t_step, "wa_expanded_per_s": wa_expanded / t_step,
+            "wa_covered_per_s": wa_covered / t_step,
+            "wa_resolved_per_step": wa_resolved, "wa_expanded_per_step": wa_expanded,
+            "wa_covered_per_step": wa_covered, "invalid": n_invalid,
             "wa_closed_form_per_step": wa_closed,
+            "wa_note": ("resolved = counted exactly on the GPU (closed forms included), expanded = of those, "
+                        "expanded lane by lane, covered = sum over candidates (count sharing)"),
             "hbm_gbs": hbm_bytes / t_step / 1e9, "roofline": roofline,
             "roofline_by_region": {k: {kk: v[kk] for kk in ("bound", "achieved", "peak", "unit", "frac", "traffic",
                                                             "ms_per_launch", "share_of_step")}
                                    for k, v in regions.items()},
-            "roofline_count": roof_count, "step_hbm_roofline": step_hbm,
+            "kernel_ms": {k: per_launch[k] for k in ("k_problem_w", "k_lane_problems", "k_model_fused")},
+            "int_pipe_ncu": int_pipe, "count_nominal_ops": roof_count, "step_hbm_roofline": step_hbm,
             "gpu_launches": launches,
             "clocks": clocks, "e2e": e2e, "gen_s": t_gen}
     if not args.no_next and args.config == 5:
         line["next_rows"] = time_next_rows(sel, gen, ev, batch, cands, args, c0, c1, dev)
     if not args.no_cpu_baseline and world == 1:
-        line["cpu_baseline"] = cpu_oracle_sample(batch, args.cpu_seconds, total)
+        keep = {}
+        line["cpu_baseline"] = cpu_oracle_sample(batch, args.cpu_seconds, total, keep)
+        if not split:
+            line["parity"] = parity_check(sel, batch, out, keep, dev, args.flags)
     print(json.dumps(line), flush=True)
+    if line.get("parity", {}).get("mismatches"):
+        sys.exit(3)
+
+
+def parity_check(sel, batch, out, keep, dev, flags):
+    """Per-run parity ("parity is checked on that subset every
+    run"): the oracle records of the cpu_baseline sample against the timed
+    step's decision, status and cycles at the same candidate indices (bit for
+    bit), and the sample's counts (W, L, S, C, U, WR) from a second, small
+    sel_evaluate on the sub-batch (slot-table problem ids).  Any mismatch
+    makes bench.py exit with status 3 after printing its line."""
+    import torch
+    idx, ref = keep["idx"], keep["ref"]
+    it = torch.from_numpy(idx).to(dev)
+    got = {k: out[k][it].cpu().numpy() for k in ("decision", "status", "cycles")}
+    sub = batch.select(idx)
+    ev2 = sel.Evaluator((sub.nests, sub.accesses, sub.launches, sub.devices), len(sub), flags, device=dev)
+    r2 = ev2.evaluate(sel._as_bytes_tensor(sub.cands, "candidate", dev), want_counts=True)
+    cnt = r2["counts"].cpu().numpy().astype(np.uint64)
+    bad = {"decision": int((got["decision"] != ref["decision"]).sum()),
+           "status": int((got["status"] != ref["status"]).sum()),
+           "cycles": int((got["cycles"].view(np.uint64) != ref["cycles"].view(np.uint64)).sum()),
+           "subset_call_decision": int((r2["decision"].cpu().numpy() != ref["decision"]).sum()),
+           "subset_call_cycles": int((r2["cycles"].cpu().numpy().view(np.uint64)
+                                      != ref["cycles"].view(np.uint64)).sum())}
+    for j, f in enumerate(("W", "L", "S", "C", "U", "WR")):
+        bad[f] = int((cnt[:, j] != ref[f]).sum())
+    del ev2
+    return {"checked": int(len(idx)), "mismatches": int(sum(bad.values())), "by_field": bad,
+            "how": ("oracle (cpu_baseline sample) vs the timed step's outputs at the same indices, bit for bit; "
+                    "counts via a second sel_evaluate on the sample")}
 
 
 def time_next_rows(sel, gen, ev, batch, cands, args, c0, c1, dev):

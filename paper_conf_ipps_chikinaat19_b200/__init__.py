@@ -23,11 +23,14 @@ from ._lib import (DECISION_CPU, DECISION_GPU, DECISION_INVALID, SEL_EINTERNAL, 
                    SEL_ERANGE, SEL_F_MATCH_ANY, SEL_F_NO_DEDUP, SEL_OK, SelError)
 
 __all__ = ["load_device_params", "workspace_size", "DeviceTables", "count_transactions", "predict_gpu_cycles",
-           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "profile_read_region", "PROF_PLAN", "PROF_COUNT", "PROF_MODEL", "kernel_launches",
+           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "profile_read_region", "PROF_PLAN", "PROF_COUNT", "PROF_MODEL",
+           "PROF_K_MODEL", "PROF_K_LANE", "PROF_K_PROBLEM_W", "kernel_launches",
            "Evaluator", "SelError", "SEL_F_NO_DEDUP", "SEL_F_MATCH_ANY", "DECISION_CPU", "DECISION_GPU",
            "DECISION_INVALID", "SEL_OK", "SEL_EINVAL", "SEL_ERANGE", "SEL_ELAUNCH", "SEL_EINTERNAL"]
 
-_REC_SIZE = {"device": 88, "access": 64, "nest": 88, "launch": 16, "candidate": 24, "counts": 48}
+_REC_SIZE = {"device": ctypes.sizeof(_lib.DeviceParams), "access": ctypes.sizeof(_lib.Access),
+             "nest": ctypes.sizeof(_lib.Nest), "launch": ctypes.sizeof(_lib.Launch),
+             "candidate": ctypes.sizeof(_lib.Candidate), "counts": ctypes.sizeof(_lib.Counts)}
 
 
 def _as_bytes_tensor(x, rec: str, device="cuda") -> torch.Tensor:
@@ -217,9 +220,9 @@ def read_stats(workspace: torch.Tensor, stream=None) -> dict:
     st = _lib.Stats()
     wp, _ = _ws_ptr(workspace)
     _lib.check(_lib.lib().sel_read_stats(wp, ctypes.byref(st), _stream(stream)))
-    return {k: int(getattr(st, k)) for k in ("n_candidates", "n_problems", "wa_analysed", "wa_covered",
+    return {k: int(getattr(st, k)) for k in ("n_candidates", "n_problems", "wa_resolved", "wa_covered",
                                              "n_invalid", "wa_closed_form", "wa_arith_lanes", "wa_residue_classes",
-                                             "alg_lane_ops")}
+                                             "alg_lane_ops", "wa_expanded")}
 
 
 def profile_enable(on: bool = True) -> None:
@@ -233,12 +236,13 @@ def profile_read():
     return ms.value, k.value
 
 
-PROF_PLAN, PROF_COUNT, PROF_MODEL = 0, 1, 2        # sel.h SEL_PROF_*
+PROF_PLAN, PROF_COUNT, PROF_MODEL = 0, 1, 2        # sel.h SEL_PROF_*: regions
+PROF_K_MODEL, PROF_K_LANE, PROF_K_PROBLEM_W = 3, 4, 5   # single kernels
 
 
 def profile_read_region(region: int):
     """-> (milliseconds, launches) of one profiling region (PROF_PLAN,
-    PROF_COUNT, PROF_MODEL) since its last read."""
+    PROF_COUNT, PROF_MODEL) or kernel (PROF_K_*) since its last read."""
     ms, k = ctypes.c_double(), ctypes.c_uint64()
     _lib.check(_lib.lib().sel_profile_read_region(int(region), ctypes.byref(ms), ctypes.byref(k)))
     return ms.value, k.value

@@ -78,10 +78,11 @@ class Tables(ctypes.Structure):
 
 class Stats(ctypes.Structure):
     _fields_ = [("n_candidates", ctypes.c_uint64), ("n_problems", ctypes.c_uint64),
-                ("wa_analysed", ctypes.c_uint64), ("wa_covered", ctypes.c_uint64),
+                ("wa_resolved", ctypes.c_uint64), ("wa_covered", ctypes.c_uint64),
                 ("n_invalid", ctypes.c_uint64), ("wa_closed_form", ctypes.c_uint64),
                 ("wa_arith_lanes", ctypes.c_uint64), ("wa_residue_classes", ctypes.c_uint64),
-                ("alg_lane_ops", ctypes.c_uint64), ("_reserved", ctypes.c_uint64 * 7)]
+                ("alg_lane_ops", ctypes.c_uint64), ("wa_expanded", ctypes.c_uint64),
+                ("_reserved", ctypes.c_uint64 * 6)]
 
 
 RECORDS = (DeviceParams, Access, Nest, Launch, Candidate, Counts)

@@ -79,6 +79,7 @@ WsPtrs ws_ptrs(void* ws, uint64_t n, uint64_t n_nests, uint32_t flags) {
     p.prob_status = reinterpret_cast<uint8_t*>(b + L.prob_status);
     p.cand_status = reinterpret_cast<uint8_t*>(b + L.cand_status);
     p.queue = reinterpret_cast<unsigned long long*>(b + L.queue);
+    p.prob_used = reinterpret_cast<uint8_t*>(b + L.prob_used);
     p.prob_md = b + L.prob_md;
     p.cls = reinterpret_cast<uint32_t*>(b + L.cls);
     p.nest_key = reinterpret_cast<uint8_t*>(b + L.nest_key);
@@ -163,7 +164,7 @@ int sel_count_transactions_part(const sel_candidate* c, uint64_t n, const sel_ta
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     const WsPtrs w = ws_ptrs(ws, n, t->n_nests, flags);
     if (int r = plan_and_count(c, n, t, w, flags, s, part, n_parts)) return r;
-    cudaError_t e = launch_gather_counts(n, w, out, status, s);
+    cudaError_t e = launch_gather_counts(c, n, *t, w, out, status, s);
     if (e != cudaSuccess) return cuda_fail(e, "gather");
     return SEL_OK;
 }
@@ -245,6 +246,7 @@ int sel_read_stats(const void* ws, sel_stats* out, sel_stream_t stream) {
     cudaError_t e = cudaMemcpyAsync(out, ws, sizeof(sel_stats), cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return cuda_fail(e, "sel_read_stats");
+    out->wa_expanded = out->wa_resolved - out->wa_closed_form - out->wa_arith_lanes - out->wa_residue_classes;
     return SEL_OK;
 }
 

@@ -1434,7 +1434,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
     const uint32_t ncls = direct ? a.hdr->n_cls : 1u;
     const uint64_t qb = a.hdr->small_begin, qe = a.hdr->small_end;
     const uint64_t ub = qb / ncls, ue = (qe + ncls - 1) / ncls;
-    uint32_t sK = 0, sH = 0;                                // statistics: WAs by path
+    unsigned long long sK = 0, sH = 0;                      // statistics: WAs by path (64-bit: ADVICE r01)
     unsigned long long sW = 0, sOps = 0;
     for (uint64_t t0 = ub + uint64_t(blockIdx.x) * kLaneTile; t0 < ue; t0 += uint64_t(gridDim.x) * kLaneTile) {
         const uint32_t nt = uint32_t(umin64(kLaneTile, ue - t0));
@@ -1526,7 +1526,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                             for (uint32_t c = 0; c < kLaneGrp; c++)
                                 if ((vmask >> c) & 1u) {
                                     lane_uniform(rc[c], Mk, g != 0, tc, z[c]);
-                                    sK += WR[c] * Mk;
+                                    sK += uint64_t(WR[c]) * Mk;
                                     z[c].W += WR[c] * Mk;
                                 }
                         } else if (d <= 2 && ac.elem_bytes >= 4 && a.residue_classes) {
@@ -1535,7 +1535,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                             for (uint32_t c = 0; c < kLaneGrp; c++)
                                 if ((vmask >> c) & 1u) {
                                     lane_hist_eval(hcol, ac, uint32_t(nest.P0), B[c], WR[c], rc[c], tc, z[c]);
-                                    sH += WR[c] * Mk;
+                                    sH += uint64_t(WR[c]) * Mk;
                                     z[c].W += WR[c] * Mk;
                                 }
                         } else {
@@ -1583,12 +1583,15 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
         }
         __syncthreads();                                    // s_order / s_cnt are rewritten by the next tile
     }
-    const uint32_t K = __reduce_add_sync(kFull, sK), H = __reduce_add_sync(kFull, sH);
-    unsigned long long Wt = sW;
-    for (int o = 16; o; o >>= 1) Wt += __shfl_xor_sync(kFull, Wt, o);
-    if (K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, (unsigned long long)K);
-    if (H && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, (unsigned long long)H);
-    if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_analysed, Wt);
+    unsigned long long K = sK, H = sH, Wt = sW;
+    for (int o = 16; o; o >>= 1) {
+        K += __shfl_xor_sync(kFull, K, o);
+        H += __shfl_xor_sync(kFull, H, o);
+        Wt += __shfl_xor_sync(kFull, Wt, o);
+    }
+    if (K && lane == 0) atomicAdd((unsigned long long*)&a.hdr->stats.wa_closed_form, K);
+    if (H && lane == 1) atomicAdd((unsigned long long*)&a.hdr->stats.wa_residue_classes, H);
+    if (Wt && lane == 2) atomicAdd((unsigned long long*)&a.hdr->stats.wa_resolved, Wt);
     for (int o = 16; o; o >>= 1) sOps += __shfl_xor_sync(kFull, sOps, o);
     if (sOps && lane == 3) atomicAdd((unsigned long long*)&a.hdr->stats.alg_lane_ops, sOps);
 }
@@ -1778,7 +1781,9 @@ static void launch_mode(const CountArgs& a, cudaStream_t s) {
         g_lane = persistent_grid(k_lane_problems<MODE>, kLaneThreads, kLaneSmem);
     }
     if (MODE != 0) {
+        prof_begin(SEL_PROF_K_LANE, s);
         k_lane_problems<MODE><<<g_lane, kLaneThreads, lane_smem, s>>>(a);
+        prof_end(SEL_PROF_K_LANE, s);
         k_queue<MODE><<<g_queue, SEL_COUNT_THREADS, 0, s>>>(a);
         note_launch(2);
     }

@@ -16,7 +16,7 @@ constexpr uint32_t kNoProblem = 0xffffffffu;
 constexpr int kSlots = 8;              // distinct B classes shared per nest before overflow
 constexpr uint32_t kClsMax = 1024;     // launch tables up to this size use direct problem ids
 constexpr int kCntStride = 6;          // per problem: W, L, S, C, U (atomic), M_it (closed form)
-constexpr size_t kProbModelBytes = 96; // per problem: the candidate-independent part of a4-a6 (sel_model.cu)
+constexpr size_t kProbModelBytes = 112; // per problem: the candidate-independent part of a4 (sel_model.cu)
 
 // ------------------------------------------------------------------ workspace
 // All offsets are 256-byte aligned.  Sized for the worst case of one counting
@@ -35,13 +35,16 @@ struct WsHeader {
     unsigned int direct;               // 1: problem id = nest * n_cls + class of the launch (k_classes)
     unsigned int n_cls;                // distinct B classes of the launch table (direct mode)
     unsigned long long n_nests_scan;   // nests scanned by the slot-table path (0 in direct mode)
-    unsigned long long _pad[4];
+    unsigned long long n_big;          // direct mode: problems counted through the WA prefix (k_count)
+    unsigned int skip_scan;            // direct mode without big problems: the W prefix is all zero
+    unsigned int _pad1;
+    unsigned long long _pad[2];
 };
 static_assert(sizeof(WsHeader) == 256, "header size");
 
 struct WsLayout {
     size_t hdr, slots, nest_base, cand_pid, prob_nest, prob_B, prob_W, prob_WR, prob_cnt,
-        prob_status, cand_status, queue, prob_md, cls, nest_key, scan_tmp, total;
+        prob_status, cand_status, queue, prob_used, prob_md, cls, nest_key, scan_tmp, total;
 };
 
 __host__ __device__ inline size_t ws_align(size_t x) { return (x + 255) & ~size_t(255); }
@@ -68,6 +71,7 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
     L.prob_status = o; o = ws_align(o + n);
     L.cand_status = o; o = ws_align(o + n);
     L.queue = o;      o = ws_align(o + n * sizeof(uint64_t));
+    L.prob_used = o;  o = ws_align(o + n);
     L.prob_md = o;    o = ws_align(o + n * kProbModelBytes);
     L.cls = o;        o = ws_align(o + 2 * kClsMax * sizeof(uint32_t));
     L.nest_key = o;   o = ws_align(o + n);

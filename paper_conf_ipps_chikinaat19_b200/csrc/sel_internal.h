@@ -22,6 +22,7 @@ struct WsPtrs {
     uint8_t* prob_status;
     uint8_t* cand_status;
     unsigned long long* queue;       // (problem << 32 | first WA) handed from the lane to the warp kernel
+    uint8_t* prob_used;              // direct mode: big problem referenced by a candidate (k_mark_big)
     void* prob_md;                   // per problem: ProbModel (sel_model.cu)
     uint32_t* cls;                   // [kClsMax] class index per launch, [kClsMax..) B class per index
     uint8_t* nest_key;               // direct mode: shape key per nest (k_problem_w -> k_lane_problems)
@@ -48,7 +49,8 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
 // sel_model.cu
 int n_device_sets();
 cudaError_t load_device_params(const sel_device_params* host, int n);
-cudaError_t launch_gather_counts(uint64_t n, const WsPtrs& w, sel_counts* out, uint8_t* status,
+cudaError_t launch_gather_counts(const sel_candidate* cands, uint64_t n, const sel_tables& t, const WsPtrs& w,
+                                 sel_counts* out, uint8_t* status,
                                  cudaStream_t s);
 cudaError_t launch_model_fused(const sel_candidate* cands, uint64_t n, const sel_tables& t, const WsPtrs& w,
                                uint8_t* decision, double* cycles, double* t_gpu, sel_counts* counts,

@@ -20,7 +20,8 @@ namespace sel {
 // x[n] = total.  n is read from *n_dev when given (device-side count).
 __global__ void __launch_bounds__(kScanThreads) k_scan_reduce(const unsigned long long* x, uint64_t n_host,
                                                               const unsigned long long* n_dev,
-                                                              unsigned long long* partial) {
+                                                              unsigned long long* partial, const unsigned* skip) {
+    if (skip && *skip) return;
     const uint64_t n = n_dev ? *n_dev : n_host;
     const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
     unsigned long long s = 0;
@@ -43,7 +44,9 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_reduce(const unsigned lon
 
 // single block: exclusive scan of the per-block partial sums
 __global__ void __launch_bounds__(1024) k_scan_partials(unsigned long long* partial, uint64_t nb_host,
-                                                        uint64_t n_host, const unsigned long long* n_dev) {
+                                                        uint64_t n_host, const unsigned long long* n_dev,
+                                                        const unsigned* skip) {
+    if (skip && *skip) return;
     const uint64_t n = n_dev ? *n_dev : n_host;
     uint64_t nb = (n + kScanItems - 1) / kScanItems;
     if (nb > nb_host) nb = nb_host;
@@ -80,7 +83,8 @@ __global__ void __launch_bounds__(1024) k_scan_partials(unsigned long long* part
 
 __global__ void __launch_bounds__(kScanThreads) k_scan_down(unsigned long long* x, uint64_t n_host,
                                                             const unsigned long long* n_dev,
-                                                            const unsigned long long* partial) {
+                                                            const unsigned long long* partial, const unsigned* skip) {
+    if (skip && *skip) return;
     const uint64_t n = n_dev ? *n_dev : n_host;
     const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
     if (begin > n) return;
@@ -117,12 +121,14 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_down(unsigned long long* 
     if (last >= n && threadIdx.x == 0 && n < last) x[n] = partial[blockIdx.x + 1];
 }
 
+// skip (device flag, optional): set by the plan when every x[i] is zero -- the
+// prefix is then all zero and only x[n] = 0 must be written (k_drop_unused)
 static cudaError_t scan_u64(unsigned long long* x, uint64_t n_max, const unsigned long long* n_dev,
-                            unsigned long long* partial, cudaStream_t s) {
+                            unsigned long long* partial, cudaStream_t s, const unsigned* skip = nullptr) {
     const uint64_t nb = (n_max + kScanItems) / kScanItems;     // covers index n_max as well
-    k_scan_reduce<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial);
-    k_scan_partials<<<1, 1024, 0, s>>>(partial, nb, n_max, n_dev);
-    k_scan_down<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial);
+    k_scan_reduce<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
+    k_scan_partials<<<1, 1024, 0, s>>>(partial, nb, n_max, n_dev, skip);
+    k_scan_down<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
     note_launch(3);
     return cudaGetLastError();
 }
@@ -131,9 +137,9 @@ static cudaError_t scan_u64(unsigned long long* x, uint64_t n_max, const unsigne
 // Direct problem ids (launch tables of <= kClsMax entries whose nests x
 // classes fit the workspace): the distinct B classes of the launch table,
 // sorted, give every launch a class index, and problem = nest * n_cls +
-// class index -- deterministic, no slot table, no second pass over the
-// candidates.  Problems no candidate refers to keep prob_nest = kNoProblem
-// and are skipped.  One block; O(n_launches^2) comparisons.
+// class index -- deterministic, no slot table, no pass over the candidates
+// (k_problem_w sets up every nest x class problem; k_model_tile derives the
+// id of each candidate).  One block; O(n_launches^2) comparisons.
 __global__ void __launch_bounds__(1024) k_classes(sel_tables t, uint64_t n, uint64_t n_nests, int dedup,
                                                   WsHeader* hdr, uint32_t* cls) {
     __shared__ uint32_t s_bc[kClsMax];
@@ -184,8 +190,10 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
                                                 uint32_t* prob_B, uint32_t* cand_pid, const WsHeader* hdr,
                                                 const uint32_t* cls) {
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
-    const bool direct = dedup && hdr->direct;
-    const uint32_t ncls = hdr->n_cls;
+    // direct mode: the model kernel derives problem ids and validates V1-V2
+    // itself, and every (nest, class) pair is a problem -- no pass over the
+    // candidates here
+    if (dedup && hdr->direct) return;
     for (uint64_t base = uint64_t(blockIdx.x) * blockDim.x; base < n; base += stride) {
         const uint64_t c = base + threadIdx.x;
         const bool in = c < n;
@@ -194,18 +202,6 @@ __global__ void __launch_bounds__(256) k_insert(const sel_candidate* __restrict_
         const sel_candidate cd = cands[c];
         const uint8_t st = validate_candidate(cd, t, n_sets);
         cand_status[c] = st;
-        if (direct) {
-            const uint32_t ci = st ? 0u : cls[cd.launch_id];
-            const uint32_t pid = st ? kNoProblem : cd.nest_id * ncls + ci;
-            cand_pid[c] = pid;
-            // identical values from every sharer: one write per distinct problem of the warp
-            const unsigned peers = __match_any_sync(inmask, pid);
-            if (!st && int(threadIdx.x & 31) == __ffs(peers) - 1) {
-                prob_nest[pid] = cd.nest_id;
-                prob_B[pid] = cls[kClsMax + ci];
-            }
-            continue;
-        }
         if (!dedup) {
             cand_pid[c] = st ? kNoProblem : uint32_t(c);          // kNoProblem <=> candidate invalid (all modes)
             prob_nest[c] = st ? kNoProblem : cd.nest_id;
@@ -297,7 +293,7 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 // The counters of a small problem with W > 0 are not zeroed here: in a
 // single-part call the lane kernel thread that counts it STORES its sums
 // (k_queue adds the handed-over accesses afterwards).
-__device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
+__device__ __forceinline__ bool problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
                                               const uint32_t* prob_B, unsigned long long* prob_W,
                                               unsigned long long* prob_WR, uint8_t* prob_status,
                                               unsigned long long* prob_cnt, int lane_ok, bool one_part) {
@@ -306,7 +302,7 @@ __device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, 
         for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
         prob_W[q] = 0;
         prob_WR[q] = 0;
-        return;
+        return false;
     }
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
@@ -317,16 +313,22 @@ __device__ __forceinline__ void problem_w_one(uint64_t q, const sel_nest& nest, 
     prob_W[q] = small ? 0ull : W;
     if (!(small && W != 0 && one_part))
         for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
+    return !small && W != 0;                 // counted through the WA prefix (k_count)
 }
 
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
-                                                   unsigned long long* prob_cnt, int lane_ok, uint8_t* nest_key) {
+                                                   unsigned long long* prob_cnt, int lane_ok, uint8_t* nest_key,
+                                                   uint32_t* prob_nest_w, uint32_t* prob_B_w, const uint32_t* cls,
+                                                   uint8_t* prob_used) {
     const uint64_t nq = hdr->n_problems;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     if (hdr->direct) {
-        // direct ids: the problems of nest i are i * n_cls + [0, n_cls).  A warp
+        // direct ids: the problems of nest i are i * n_cls + [0, n_cls), every
+        // one of them counted (direct mode requires n_nests * n_cls <= n, so
+        // at most one problem per candidate; a big problem no candidate refers
+        // to is dropped again by k_mark_big / k_drop_unused).  A warp
         // takes 32 nests (lane = nest), checks the concatenation of their access
         // lists 32 accesses at a time (lane = access: the descriptor loads are
         // independent and, for consecutive nests, contiguous), reduces each
@@ -339,18 +341,14 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
         const uint64_t nn = ncls ? nq / ncls : 0;
         const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
         const uint64_t nwarps = uint64_t(gridDim.x) * (blockDim.x >> 5);
-        uint32_t used = 0;
+        uint32_t used = 0, big = 0;
         for (uint64_t i0 = (uint64_t(blockIdx.x) * (blockDim.x >> 5) + wib) * 32; i0 < nn; i0 += nwarps * 32) {
             const uint64_t i = i0 + lane;
-            uint32_t um = 0;
             sel_nest nest{};
             uint8_t pre = SEL_EINVAL;
             if (i < nn) {
-                for (uint32_t c = 0; c < ncls; c++) um |= (prob_nest[i * ncls + c] != kNoProblem ? 1u : 0u) << (c & 31u);
-                if (um || ncls > 32) {
-                    nest = t.nests[i];
-                    pre = nest_precheck(nest, t.n_accesses);
-                }
+                nest = t.nests[i];
+                pre = nest_precheck(nest, t.n_accesses);
             }
             const uint32_t na = pre == SEL_OK ? nest.n_access : 0u;
             uint32_t incl = na;                                 // inclusive prefix of the access counts
@@ -428,16 +426,20 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                 const uint8_t st = nest_status(pre, s_flags[wib][lane], P, M_it);
                 for (uint32_t c = 0; c < ncls; c++) {
                     const uint64_t q = i * ncls + c;
-                    const bool u = c < 32 ? ((um >> c) & 1u) : prob_nest[q] != kNoProblem;
-                    used += u ? 1u : 0u;
-                    problem_w_one(q, nest, u ? st : uint8_t(SEL_EINVAL), st == SEL_OK ? M_it : 0ull, prob_B, prob_W,
-                                  prob_WR, prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
+                    used++;
+                    prob_nest_w[q] = uint32_t(i);
+                    prob_B_w[q] = cls[kClsMax + c];
+                    prob_used[q] = 0;
+                    big += problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, prob_B, prob_W, prob_WR,
+                                         prob_status, prob_cnt, lane_ok, hdr->n_parts == 1) ? 1u : 0u;
                 }
             }
             __syncwarp();
         }
         used = __reduce_add_sync(kFull, used);
+        big = __reduce_add_sync(kFull, big);
         if ((threadIdx.x & 31) == 0 && used) atomicAdd((unsigned long long*)&hdr->stats.n_problems, (unsigned long long)used);
+        if ((threadIdx.x & 31) == 0 && big) atomicAdd((unsigned long long*)&hdr->n_big, (unsigned long long)big);
         return;
     }
     // grid-stride: the grid is sized for the candidates, the problems (known on
@@ -455,6 +457,50 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
     }
 }
 
+// Direct mode with big problems (counted warp-access by warp-access through
+// the prefix): mark the ones some valid candidate refers to, then drop the
+// others from the prefix (unreferenced small problems are left in: their
+// closed-form counting costs O(accesses) per nest).  Both return at once when
+// the batch has no big problem (c5) -- a launch each, no pass over the data.
+__global__ void __launch_bounds__(256) k_mark_big(const sel_candidate* __restrict__ cands, uint64_t n, sel_tables t,
+                                                  int n_sets, WsHeader* hdr, const uint32_t* cls,
+                                                  const unsigned long long* prob_W, uint8_t* prob_used) {
+    if (!hdr->direct || hdr->n_big == 0) return;
+    const uint32_t ncls = hdr->n_cls;
+    for (uint64_t c = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; c < n; c += uint64_t(gridDim.x) * blockDim.x) {
+        const sel_candidate cd = cands[c];
+        if (validate_candidate(cd, t, n_sets)) continue;
+        const uint64_t q = uint64_t(cd.nest_id) * ncls + cls[cd.launch_id];
+        if (prob_W[q] != 0 && !prob_used[q]) prob_used[q] = 1;
+    }
+}
+__global__ void __launch_bounds__(256) k_drop_unused(WsHeader* hdr, unsigned long long* prob_W,
+                                                     unsigned long long* prob_WR, unsigned long long* prob_cnt,
+                                                     uint8_t* prob_status, const uint8_t* prob_used) {
+    if (!hdr->direct) return;
+    const uint64_t nq = hdr->n_problems;
+    if (hdr->n_big == 0) {                        // no W in the prefix: all-zero, skip the scan
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            hdr->skip_scan = 1;
+            prob_W[nq] = 0;
+        }
+        return;
+    }
+    uint32_t dropped = 0;
+    for (uint64_t q = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; q < nq; q += uint64_t(gridDim.x) * blockDim.x) {
+        if (prob_W[q] != 0 && !prob_used[q]) {
+            prob_W[q] = 0;
+            prob_WR[q] = 0;
+            prob_cnt[q * kCntStride + 5] = 0;
+            prob_status[q] = SEL_EINVAL;             // not counted; no candidate refers to it
+            dropped++;
+        }
+    }
+    dropped = __reduce_add_sync(kFull, dropped);
+    if ((threadIdx.x & 31) == 0 && dropped)
+        atomicAdd((unsigned long long*)&hdr->stats.n_problems, 0ull - (unsigned long long)dropped);
+}
+
 // slice [total*part/n_parts, total*(part+1)/n_parts) of the problem work space
 // (one huge candidate's warp-accesses split R ways)
 __global__ void k_plan_stats(WsHeader* hdr, const unsigned long long* prefix) {
@@ -463,7 +509,7 @@ __global__ void k_plan_stats(WsHeader* hdr, const unsigned long long* prefix) {
     const uint64_t e = uint64_t(total * (hdr->part + 1) / hdr->n_parts);
     hdr->w_begin = b;
     hdr->w_end = e;
-    hdr->stats.wa_analysed = e - b;               // + the small problems' W (k_lane_problems)
+    hdr->stats.wa_resolved = e - b;               // + the small problems' W (k_lane_problems)
     const unsigned __int128 nq = hdr->n_problems;
     hdr->small_begin = uint64_t(nq * hdr->part / hdr->n_parts);
     hdr->small_end = uint64_t(nq * (hdr->part + 1) / hdr->n_parts);
@@ -480,10 +526,6 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
     if (e != cudaSuccess) return e;
     if (dedup && n_nests) {
         e = cudaMemsetAsync(w.slots, 0, n_nests * kSlots * sizeof(uint32_t), s);
-        if (e != cudaSuccess) return e;
-        // direct mode: problem ids no candidate refers to stay kNoProblem
-        const uint64_t ids = n_nests * (t.n_launches < kClsMax ? t.n_launches : kClsMax);
-        e = cudaMemsetAsync(w.prob_nest, 0xff, (ids < n ? ids : n) * sizeof(uint32_t), s);
         if (e != cudaSuccess) return e;
     }
     k_classes<<<1, 1024, 0, s>>>(t, n, n_nests, dedup ? 1 : 0, w.hdr, w.cls);
@@ -502,13 +544,20 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
         note_launch();
     }
     k_finalize_plan<<<1, 1, 0, s>>>(w.hdr, w.nest_base, n_nests, n, dedup ? 1 : 0, part, n_parts);
+    prof_begin(SEL_PROF_K_PROBLEM_W, s);
     k_problem_w<<<gb, 256, 0, s>>>(t, w.hdr, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR,
                                                           w.prob_status, w.prob_cnt,
                                                           (flags & (SEL_F_MATCH_ANY | SEL_F_EXPAND_ALL |
                                                                     SEL_F_WARP_PROBLEMS)) ? 0 : 1,
-                                                          w.nest_key);
+                                                          w.nest_key, w.prob_nest, w.prob_B, w.cls, w.prob_used);
+    prof_end(SEL_PROF_K_PROBLEM_W, s);
     note_launch(2);
-    if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s)) != cudaSuccess) return e;
+    if (dedup) {
+        k_mark_big<<<148u * 8, 256, 0, s>>>(cands, n, t, n_sets, w.hdr, w.cls, w.prob_W, w.prob_used);
+        k_drop_unused<<<148u * 8, 256, 0, s>>>(w.hdr, w.prob_W, w.prob_WR, w.prob_cnt, w.prob_status, w.prob_used);
+        note_launch(2);
+    }
+    if ((e = scan_u64(w.prob_W, n, &w.hdr->n_problems, w.scan_tmp, s, &w.hdr->skip_scan)) != cudaSuccess) return e;
     k_plan_stats<<<1, 1, 0, s>>>(w.hdr, w.prob_W);
     note_launch();
     prof_end(SEL_PROF_PLAN, s);

@@ -4,8 +4,13 @@ Candidates are independent: each rank evaluates a contiguous
 range of the candidate index space with no data-path exchange; the only
 collective is the all-gather of the per-candidate decisions the north star
 asks for (NCCL over NVLink / NVSwitch on a GPU box, gloo in the CPU tests).
-Ranges are padded to a common length so a single ``all_gather_into_tensor``
-suffices; padding bytes are dropped after the gather.  Config 4 (a few huge
+Rank r owns [r * n_pad, (r + 1) * n_pad) with n_pad = ceil(total / world), so
+the ranks' slots of ONE preallocated buffer hold every decision in candidate
+order: each rank evaluates straight into its slot and a single in-place
+``all_gather_into_tensor`` fills the rest (``DecisionGather``; no
+allocation, zero-fill or concatenation per step).  ``weighted_ranges`` cuts
+the index space at equal shares of a per-candidate work prefix instead
+(cut points at k * sum(W) / R).  Config 4 (a few huge
 candidates) splits each candidate's warp-accesses instead (``evaluate_split``).
 """
 from __future__ import annotations
@@ -55,40 +60,76 @@ def _host_staged(t: torch.Tensor) -> bool:
     return t.is_cuda and dist.is_initialized() and dist.get_backend() == "gloo"
 
 
-def shard_range(total: int, rank: int, world: int):
-    """Contiguous candidate range [c0, c1) of ``rank``; sizes differ by <= 1.
-    The c5 index interleave (device, launch, kernel in the low digits) makes
-    equal-count ranges near-equal work."""
-    base, rem = divmod(total, world)
-    c0 = rank * base + min(rank, rem)
-    return c0, c0 + base + (1 if rank < rem else 0)
-
-
 def padded_len(total: int, world: int) -> int:
     return -(-total // world)
 
 
-def gather_decisions(local: torch.Tensor, total: int, world: int, out: torch.Tensor | None = None,
-                     group=None) -> torch.Tensor:
-    """All-gather uint8 decisions of every rank's shard into a ``total``-long
-    vector in candidate order (identical on every rank)."""
+def shard_range(total: int, rank: int, world: int):
+    """Contiguous candidate range [c0, c1) of ``rank``: [r n_pad, (r+1) n_pad)
+    clipped to ``total`` (n_pad = ceil(total / world)), so rank r's padded
+    slot of the gather buffer starts at candidate r * n_pad.  The c5 index
+    interleave (device, launch, kernel in the low digits) makes equal-count
+    ranges near-equal work."""
+    n_pad = padded_len(total, world)
+    c0 = min(total, rank * n_pad)
+    return c0, min(total, c0 + n_pad)
+
+
+def weighted_ranges(prefix, world: int):
+    """Cut points of a work-balanced partition: ``prefix`` is the inclusive
+    prefix sum of per-candidate work (e.g. the closed-form W = WR * M_it of
+    each candidate), rank r gets [cut_r, cut_{r+1}) with cut_r the first
+    index whose prefix reaches r * total / world.  Contiguous, covering,
+    deterministic; ranks may be empty."""
+    import numpy as np
+    p = np.asarray(prefix)
+    n = len(p)
+    total = int(p[-1]) if n else 0
+    cuts = [0]
+    for r in range(1, world):
+        cuts.append(int(np.searchsorted(p, (total * r + world - 1) // world, side="left")) if total else n * r // world)
+    cuts.append(n)
+    cuts = [min(max(c, cuts[i - 1] if i else 0), n) for i, c in enumerate(cuts)]
+    return [(cuts[r], cuts[r + 1]) for r in range(world)]
+
+class DecisionGather:
+    """Preallocated all-gather of the u8 decisions.  ``slot`` is
+    this rank's shard inside the gather buffer: pass it as the decision output
+    of ``sel_evaluate`` and ``gather()`` runs one in-place
+    ``all_gather_into_tensor`` (the send buffer IS the rank's chunk of the
+    receive buffer); ``gather()[:total]`` is every decision in candidate
+    order, identical on every rank.  Padding bytes (past ``total``) are set to
+    SEL_DECISION_INVALID once, at construction."""
+
+    def __init__(self, total: int, world: int, rank: int, device, group=None):
+        self.total, self.world, self.rank, self.group = total, world, rank, group
+        self.n_pad = padded_len(total, world)
+        self.buf = torch.full((self.n_pad * world,), 0xFF, dtype=torch.uint8, device=device)
+        c0, c1 = shard_range(total, rank, world)
+        self.chunk = self.buf[rank * self.n_pad:(rank + 1) * self.n_pad]
+        self.slot = self.chunk[: c1 - c0]
+        self._host = torch.empty(self.n_pad * world, dtype=torch.uint8) if _host_staged(self.buf) else None
+
+    def gather(self) -> torch.Tensor:
+        if self.world > 1:
+            if self._host is not None:
+                dist.all_gather_into_tensor(self._host, self.chunk.cpu(), group=self.group)
+                self.buf.copy_(self._host)
+            else:
+                dist.all_gather_into_tensor(self.buf, self.chunk, group=self.group)
+        return self.buf[: self.total]
+
+
+def gather_decisions(local: torch.Tensor, total: int, world: int, group=None) -> torch.Tensor:
+    """All-gather uint8 decisions of every rank's shard (``shard_range``) into a
+    ``total``-long vector in candidate order (identical on every rank).  A
+    convenience that copies ``local`` into a fresh ``DecisionGather``; the hot
+    loop evaluates into ``DecisionGather.slot`` directly."""
     if world == 1:
         return local
-    n_pad = padded_len(total, world)
-    buf = torch.zeros(n_pad, dtype=torch.uint8, device=local.device)
-    buf[: local.numel()].copy_(local)
-    full = torch.empty(n_pad * world, dtype=torch.uint8, device=local.device) if out is None else out
-    if _host_staged(buf):
-        hfull = torch.empty(n_pad * world, dtype=torch.uint8)
-        dist.all_gather_into_tensor(hfull, buf.cpu(), group=group)
-        full.copy_(hfull)
-    else:
-        dist.all_gather_into_tensor(full, buf, group=group)
-    parts = []
-    for r in range(world):
-        c0, c1 = shard_range(total, r, world)
-        parts.append(full[r * n_pad: r * n_pad + (c1 - c0)])
-    return torch.cat(parts)
+    g = DecisionGather(total, world, dist.get_rank(group), local.device, group)
+    g.slot.copy_(local)
+    return g.gather()
 
 
 def all_reduce_sum_(t: torch.Tensor, world: int, group=None) -> torch.Tensor:
@@ -104,6 +145,20 @@ def all_reduce_sum_(t: torch.Tensor, world: int, group=None) -> torch.Tensor:
     return t
 
 
+def all_reduce_max_(t: torch.Tensor, world: int, group=None) -> torch.Tensor:
+    """In-place element-wise MAX over ranks."""
+    if world == 1:
+        return t
+    if _host_staged(t) or t.dtype == torch.uint8:
+        h = t.to(torch.int32)
+        h = h.cpu() if _host_staged(t) else h
+        dist.all_reduce(h, op=dist.ReduceOp.MAX, group=group)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return t
+
+
 def evaluate_split(cands: torch.Tensor, tables, workspace: torch.Tensor, rank: int, world: int, flags: int = 0,
                    group=None) -> dict:
     """a few huge candidates, so every rank takes ALL
@@ -113,6 +168,9 @@ def evaluate_split(cands: torch.Tensor, tables, workspace: torch.Tensor, rank: i
     from . import count_transactions, predict_gpu_cycles, select
     counts, status = count_transactions(cands, tables, workspace, flags, part=rank, n_parts=world)
     all_reduce_sum_(counts, world, group)
+    # a rank whose self-check failed (SEL_EINTERNAL) contributed no counts: every
+    # rank takes the worst status, so no rank models incomplete counts
+    all_reduce_max_(status, world, group)
     cycles, t_gpu = predict_gpu_cycles(cands, tables, counts, status)
     decision = select(cands, t_gpu, status)
     return dict(counts=counts, status=status, cycles=cycles, t_gpu=t_gpu, decision=decision)

@@ -20,8 +20,26 @@ def test_shard_ranges_cover_exactly():
             for (a0, a1), (b0, b1) in zip(ranges, ranges[1:]):
                 assert a1 == b0
             sizes = [b - a for a, b in ranges]
-            assert max(sizes) - min(sizes) <= 1
-            assert max(sizes) <= D.padded_len(total, world)
+            n_pad = D.padded_len(total, world)
+            assert max(sizes) <= n_pad
+            # rank r's range starts at r * n_pad (its slot of the gather buffer) unless past the end
+            assert all(a == min(total, r * n_pad) for r, (a, _) in enumerate(ranges))
+
+
+def test_weighted_ranges_balance_work():
+    rng = np.random.default_rng(3)
+    for n, world in ((1, 1), (10, 3), (1000, 8), (12345, 4)):
+        w = rng.integers(0, 1000, n) * (rng.random(n) < 0.7)
+        w[: n // 10] *= 50                                   # a heavy head
+        p = np.cumsum(w)
+        r = D.weighted_ranges(p, world)
+        assert r[0][0] == 0 and r[-1][1] == n and all(a[1] == b[0] for a, b in zip(r, r[1:]))
+        total = int(p[-1]) if n else 0
+        share = [int(w[a:b].sum()) for a, b in r]
+        assert sum(share) == total
+        # every rank's work is within one candidate's work of the ideal share
+        assert max(share) <= total / world + w.max() + 1
+    assert D.weighted_ranges(np.zeros(5, np.int64), 2) == [(0, 2), (2, 5)]
 
 
 def _free_port():
@@ -43,6 +61,13 @@ def _worker(rank, world, port, total, q):
     # stand-in for the GPU decisions: a deterministic function of the candidate
     local = torch.from_numpy(((b.cands["nest_id"] + b.cands["device_id"]) % 3).astype(np.uint8))
     full = D.gather_decisions(local, total, w)
+    # the hot-loop form: write into the preallocated slot, gather in place (twice: reusable)
+    g = D.DecisionGather(total, w, r, torch.device("cpu"))
+    for _ in range(2):
+        g.slot.copy_(local)
+        assert torch.equal(g.gather(), full)
+    st = torch.tensor([0, 6 * rank, 0, rank], dtype=torch.uint8)
+    assert D.all_reduce_max_(st, w).tolist() == [0, 6, 0, 1]
     t = D.max_over_ranks(float(rank + 1), w, torch.device("cpu"))
     s = D.sum_over_ranks(c1 - c0, w, torch.device("cpu"))
     # config-4 partial counters: parts near 2^62 sum exactly (int64, no float staging)

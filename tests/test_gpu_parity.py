@@ -75,7 +75,7 @@ def test_c2_polybench_medium(sel, flags):
     assert_parity(g, ref, ctx="c2")
     st = g["stats"]
     assert st["n_candidates"] == 108 and st["n_problems"] == 27      # 4 device sets share counts
-    assert st["wa_analysed"] * 4 == st["wa_covered"] == int(ref["W"].sum())
+    assert st["wa_resolved"] * 4 == st["wa_covered"] == int(ref["W"].sum())
 
 
 def test_c2_split_api_matches_fused(sel):
@@ -126,6 +126,131 @@ def test_c4_full_size_sampled(sel):
     sub = {k: (v[pick] if isinstance(v, np.ndarray) else v) for k, v in g.items()}
     assert_parity(sub, ref, ctx="c4 full sampled")
     assert (g["status"] == 0).all()
+
+
+@pytest.mark.slow
+def test_c4_full_size_all(sel):
+    """All of c4 at full size (P = 2^24, 192 candidates, 4e9 warp-accesses) in
+    the bench configuration against the oracle's full brute-force expansion
+    (about 30 s on the box's host cores): the big-problem chunking of k_count
+    (WR = 2^19 > 1024) on every shape and launch."""
+    b = gen.generate(4)
+    g = run_gpu(sel, b)
+    ref = oracle.evaluate(b)
+    assert_parity(g, ref, ctx="c4 full")
+    assert (g["status"] == 0).all() and int(ref["W"].sum()) > 3 * 10 ** 9
+
+
+def _nests_with_candidates(nest_items, launches, rows, devices=None):
+    """A batch whose candidates (nest, launch, device) share the given nests
+    (gen.custom_batch makes one nest per item)."""
+    base = gen.custom_batch(nest_items, devices=devices, launches_=launches)
+    cands = np.zeros(len(rows), gen.CANDIDATE_DTYPE)
+    for i, (nest, li, dev) in enumerate(rows):
+        cands[i] = (nest, li, dev, 10 ** (3 + (i % 5)), 3e9)
+    return gen.Batch(cands, base.nests, base.accesses, launches, base.devices)
+
+
+def test_lane_multi_group_direct(sel):
+    """direct problem ids with more block-size classes
+    than the lane kernel counts in one pass (kLaneGrp), so its multi-group
+    loop (g0 = 3, 6, ...) rebuilds histograms and hands accesses to k_queue
+    per group -- with 1-2 byte elements and depth 3 (handed over) and a nest
+    of 35 accesses (the bit-31 "all remaining accesses" path)."""
+    rnd = random.Random(31)
+    Bs = [33, 40, 48, 72, 100, 200, 300, 64]            # 7 classes that 32 does not divide + the class 32
+    launches = np.zeros(len(Bs), gen.LAUNCH_DTYPE)
+    for i, B in enumerate(Bs):
+        launches[i] = (B, 65535 if i % 3 else 4, 0, 0)
+    nests = []
+    for k in range(6):
+        depth = [1, 2, 3, 1, 2, 0][k]
+        trip = [rnd.randint(3, 40) for _ in range(depth)]
+        n_acc = 35 if k == 3 else rnd.randint(2, 6)
+        acc = []
+        for j in range(n_acc):
+            e = rnd.choice([1, 2, 4, 4, 8, 8, 16])
+            d = rnd.randint(0, depth)
+            acc.append(gen.make_access(base=(1 << 30) + e * rnd.randint(0, 500) + 4096 * j,
+                                       c_par=[e * rnd.choice([0, 1, 2, 3, -1, 8, 33, 64])],
+                                       c_inner=[e * rnd.choice([0, 1, 5, 64, 1000]) for _ in range(d)],
+                                       elem_bytes=e, depth=d))
+        nests.append(dict(P0=rnd.choice([95, 333, 1000, 3000]), trip=trip, depth=depth, comp=[1.0] * (depth + 1),
+                          accesses=acc))
+    rows = [(nest, li, dev) for nest in range(len(nests)) for li in range(len(Bs)) for dev in (0, 2, 3)]
+    b = _nests_with_candidates(nests, launches, rows)
+    assert len(b.nests) * 8 <= len(b)                    # direct ids
+    ref = oracle.evaluate(b)
+    assert (ref["status"] == 0).all()
+    for flags in (0, 4, 16):
+        g = run_gpu(sel, b, flags)
+        assert_parity(g, ref, ctx=f"multi-group flags={flags}")
+        assert g["stats"]["n_problems"] == len(b.nests) * 8
+
+
+def test_direct_big_problems_referenced_or_not(sel):
+    """Direct ids with big problems (WR > 1024, counted through the warp-access
+    prefix): the ones a candidate refers to are counted exactly, a big nest
+    no candidate refers to is dropped from the prefix (k_mark_big /
+    k_drop_unused) and costs nothing."""
+    a = gen.make_access(base=1 << 30, c_par=(8,), c_inner=(8,), elem_bytes=8, depth=1)
+    big = dict(P0=1 << 17, trip=[5], comp=[1.0, 1.0], accesses=[a])
+    huge = dict(P0=1 << 30, trip=[1 << 10], comp=[1.0, 1.0], accesses=[a])     # 2^35 WAs if counted
+    small = dict(P0=300, trip=[7], comp=[1.0, 1.0], accesses=[a])
+    launches = np.zeros(2, gen.LAUNCH_DTYPE)
+    launches[0] = (128, 65535, 0, 0)
+    launches[1] = (200, 160, 0, 0)
+    rows = [(nest, li, dev) for nest in (0, 1) for li in (0, 1) for dev in (0, 1, 2, 3)]
+    b = _nests_with_candidates([small, big, huge], launches, rows)
+    ref = oracle.evaluate(b)
+    g = run_gpu(sel, b)
+    assert_parity(g, ref, ctx="direct big")
+    assert g["stats"]["n_problems"] == 4                  # nests 0, 1 x 2 classes; nest 2 dropped
+    assert g["stats"]["wa_resolved"] < 10 ** 8
+
+
+def _granular_devices(seed):
+    """Device sets with NEXT row f4's fields varied: allocation units off / on,
+    warp granularity 1-4, both transaction units."""
+    rnd = random.Random(seed)
+    d = gen.device_sets().copy()
+    for i in range(4):
+        d[i]["reg_alloc_unit"] = rnd.choice([0, 128, 256])
+        d[i]["warp_alloc_gran"] = rnd.choice([0, 1, 2, 4])
+        d[i]["smem_alloc_unit"] = rnd.choice([0, 128, 256, 1024])
+        d[i]["txn_sectors"] = i % 2
+    return d
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_f4_granularity_and_sector_transactions(sel, seed):
+    """NEXT row f4 (F4c, F4d): random launches with register and
+    shared-memory demands on device sets with allocation granularity and
+    either transaction unit, through the fused and the split API."""
+    rnd = random.Random(seed)
+    n = 800
+    launches = np.zeros(n, gen.LAUNCH_DTYPE)
+    items = []
+    for i in range(n):
+        e = rnd.choice([4, 8])
+        depth = rnd.choice([0, 1])
+        acc = [gen.make_access(base=(1 << 32) + e * rnd.randint(0, 64), c_par=[e * rnd.choice([1, 2, 33, -1])],
+                               c_inner=[e * rnd.choice([1, 64])][:depth], elem_bytes=e, depth=depth)]
+        launches[i] = (rnd.choice([32, 48, 96, 128, 200, 256, 640, 1024]), 65535,
+                       rnd.choice([0, 16, 24, 32, 37, 64, 100, 255]), rnd.choice([0, 100, 300, 4000, 20000, 50000]))
+        items.append(dict(P0=rnd.choice([20000, 70000, 150000]), trip=[rnd.randint(1, 3)][:depth], depth=depth,
+                          comp=[1.0, 2.0][: depth + 1], launch=i, device=rnd.randrange(4), accesses=acc,
+                          bytes_h2d=rnd.choice([0, 10 ** 6])))
+    bb = gen.custom_batch(items, devices=_granular_devices(seed), launches_=launches)
+    ref = oracle.evaluate(bb)
+    assert len(set(ref["abps"][ref["status"] == 0].tolist())) > 5
+    assert (ref["status"] == 3).sum() > 0 and (ref["status"] == 0).sum() > 600
+    sel.load_device_params(bb.devices)
+    try:
+        assert_parity(run_gpu(sel, bb), ref, ctx=f"f4 seed={seed}")
+        assert_parity(run_gpu(sel, bb, api="split"), ref, exact_cycles=False, ctx=f"f4 split seed={seed}")
+    finally:
+        sel.load_device_params(gen.device_sets())
 
 
 def test_c5_full_sweep_sampled(sel):
@@ -375,7 +500,7 @@ def test_uniform_flag_closed_form(sel, flags):
     else:
         assert 0 < st["wa_closed_form"] and 0 < st["wa_arith_lanes"] + st["wa_residue_classes"]
         assert (st["wa_closed_form"] + st["wa_arith_lanes"] + st["wa_residue_classes"]
-                < st["wa_analysed"])                                              # collapse(2) expands
+                < st["wa_resolved"])                                              # collapse(2) expands
 
 
 def test_closed_form_share_c5_slice(sel):
@@ -384,8 +509,8 @@ def test_closed_form_share_c5_slice(sel):
     b = gen.generate(5, 0, 200000)
     g0, g8 = run_gpu(sel, b, 0), run_gpu(sel, b, 8)
     assert (g0["counts"] == g8["counts"]).all() and (g0["cycles"] == g8["cycles"]).all()
-    assert g0["stats"]["wa_analysed"] == g8["stats"]["wa_analysed"]
-    assert g0["stats"]["wa_closed_form"] > g0["stats"]["wa_analysed"] // 2
+    assert g0["stats"]["wa_resolved"] == g8["stats"]["wa_resolved"]
+    assert g0["stats"]["wa_closed_form"] > g0["stats"]["wa_resolved"] // 2
 
 
 def _residue_class_batch(seed, n):
@@ -468,8 +593,10 @@ def test_direct_and_hashed_problem_ids_agree(sel):
     ref = oracle.evaluate(b)
     assert_parity(g_direct, ref, ctx="direct ids")
     assert_parity(g_hashed, ref, ctx="slot-table ids")
-    n = _distinct_problems(b)
-    assert g_direct["stats"]["n_problems"] == n == g_hashed["stats"]["n_problems"]
+    # direct ids count every (nest, class) pair of the tables; the
+    # slot table only the pairs the candidates refer to
+    assert g_direct["stats"]["n_problems"] == len(b.nests) * 3
+    assert g_hashed["stats"]["n_problems"] == _distinct_problems(b)
 
 
 def test_direct_ids_sparse_nests(sel):

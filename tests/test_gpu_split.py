@@ -47,7 +47,7 @@ def _parts(sel, b, n_parts, flags=0):
     full, st_full = sel.count_transactions(cands, ev.tables, ev.workspace, flags)
     full = full.cpu().numpy().astype(np.uint64)
     st_full = st_full.cpu().numpy()
-    total = sel.read_stats(ev.workspace)["wa_analysed"]
+    total = sel.read_stats(ev.workspace)["wa_resolved"]
     acc = np.zeros_like(full)
     sizes = []
     for p in range(n_parts):
@@ -57,7 +57,7 @@ def _parts(sel, b, n_parts, flags=0):
         if p > 0:
             assert (c[:, 5] == 0).all(), "warp_reps must come from part 0 only"
         acc += c
-        sizes.append(sel.read_stats(ev.workspace)["wa_analysed"])
+        sizes.append(sel.read_stats(ev.workspace)["wa_resolved"])
     # the parts tile the work: big problems by equal slices of the WA prefix, small
     # problems (counted one per lane) by problem-index ranges
     assert sum(sizes) == total

@@ -68,10 +68,10 @@ def test_workspace_size_monotone():
     b = L.sel_workspace_size(2000, 10, 0)
     c = L.sel_workspace_size(1000, 10, 1)
     assert 0 < a < b and c < a
-    # the c5 sweep (10^8 candidates) plans in well under a tenth of the 180 GB of HBM:
-    # ~183 B per candidate, sized for the worst case of one problem per candidate
-    # (per problem: counts 48 B, model inputs 96 B, W / WR / nest / B / status 25 B)
-    assert L.sel_workspace_size(10 ** 8, 3125000, 0) < 19 * 10 ** 9
+    # the c5 sweep (10^8 candidates) plans in an eighth of the 180 GB of HBM:
+    # ~217 B per candidate, sized for the worst case of one problem per candidate
+    # (per problem: counts 48 B, model inputs 128 B, W / WR / nest / B / status / used 26 B)
+    assert L.sel_workspace_size(10 ** 8, 3125000, 0) < 23 * 10 ** 9
 
 
 def test_product_does_not_import_oracle():

@@ -83,6 +83,7 @@ WsPtrs ws_ptrs(void* ws, uint64_t n, uint64_t n_nests, uint32_t flags) {
     p.prob_md = b + L.prob_md;
     p.cls = reinterpret_cast<uint32_t*>(b + L.cls);
     p.nest_key = reinterpret_cast<uint8_t*>(b + L.nest_key);
+    p.lane_info = reinterpret_cast<uint2*>(b + L.lane_info);
     p.scan_tmp = reinterpret_cast<unsigned long long*>(b + L.scan_tmp);
     return p;
 }

@@ -76,6 +76,8 @@ struct CountArgs {
     uint32_t residue_classes;           // whole arithmetic-lane warp-reps by residue classes (count_hist)
     unsigned long long* queue;          // small problems handed from k_lane_problems to k_queue
     const uint8_t* nest_key;            // direct mode: shape key per nest (k_problem_w)
+    const uint2* lane_info;             // direct mode: per nest (M_it, mask of classes < 32 counted here)
+    const uint32_t* cls_B;              // direct mode: B class of each class index
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -1480,9 +1482,14 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                 uint32_t B[kLaneGrp], WR[kLaneGrp], hm[kLaneGrp];
                 RepClasses rc[kLaneGrp];
                 LaneSums z[kLaneGrp];
-                uint32_t vmask = 0;
+                uint32_t vmask = 0, rc_wr = 0;          // rc_wr: WR of these classes still to take from rc
+                uint64_t Mit = 0;
                 sel_nest nest{};
                 if (has) {
+                    // direct ids: one 8-byte per-nest record (k_problem_w) says which classes are
+                    // small, valid and non-empty, and gives M_it; WR follows from the warp-rep classes
+                    const uint2 li = direct ? a.lane_info[u] : make_uint2(0u, 0u);
+                    Mit = li.x;
 #pragma unroll
                     for (uint32_t c = 0; c < kLaneGrp; c++) {
                         hm[c] = 0u;
@@ -1490,13 +1497,23 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                         B[c] = 0u;
                         WR[c] = 0u;
                         rc[c] = RepClasses{0ull, 0ull, 0u, 0u};
-                        const uint64_t q = u * ncls + g0 + c;
-                        if (g0 + c < ncls && q >= qb && q < qe && a.prefix[q + 1] == a.prefix[q]) {
+                        const uint32_t ci = g0 + c;
+                        const uint64_t q = u * ncls + ci;
+                        if (ci >= ncls || q < qb || q >= qe) continue;
+                        if (direct && ci < 32) {
+                            if ((li.y >> ci) & 1u) {
+                                vmask |= 1u << c;
+                                rc_wr |= 1u << c;
+                                B[c] = a.cls_B[ci];
+                            }
+                        } else if (a.prefix[q + 1] == a.prefix[q]) {
                             const uint64_t WR64 = a.prob_WR[q];
-                            if (WR64 * a.prob_cnt[q * kCntStride + 5]) {      // small, valid, W > 0
+                            const uint64_t M = a.prob_cnt[q * kCntStride + 5];
+                            if (WR64 * M) {                                   // small, valid, W > 0
                                 vmask |= 1u << c;
                                 WR[c] = uint32_t(WR64);
                                 B[c] = a.prob_B[q];
+                                Mit = M;
                             }
                         }
                     }
@@ -1505,7 +1522,11 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                     nest = a.nests[direct ? uint32_t(u) : a.prob_nest[u]];
 #pragma unroll
                     for (uint32_t c = 0; c < kLaneGrp; c++)
-                        if ((vmask >> c) & 1u) rc[c] = rep_classes(nest.P0, B[c]);
+                        if ((vmask >> c) & 1u) {
+                            rc[c] = rep_classes(nest.P0, B[c]);
+                            if ((rc_wr >> c) & 1u)
+                                WR[c] = uint32_t(rc[c].n32 + rc[c].nA) + (rc[c].lanesR ? 1u : 0u);
+                        }
                     const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
                                    T2 = uint32_t(eff_trip(nest.trip[2]));
                     const sel_access* ap = a.acc + nest.access_off;
@@ -1547,7 +1568,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                     for (uint32_t c = 0; c < kLaneGrp; c++) {
                         if (!((vmask >> c) & 1u)) continue;
                         const uint64_t q = u * ncls + g0 + c;
-                        sW += uint64_t(WR[c]) * a.prob_cnt[q * kCntStride + 5];
+                        sW += uint64_t(WR[c]) * Mit;
                         sOps += z[c].ops;
                         {   // the only writer so far (k_problem_w leaves these counters unzeroed): store
                             unsigned long long* pc = a.prob_cnt + q * kCntStride;
@@ -1797,7 +1818,7 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
                 (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u,
-                w.queue, w.nest_key};
+                w.queue, w.nest_key, w.lane_info, w.cls + kClsMax};
     prof_before_count(s);
     if (mode == 0) launch_mode<0>(a, s);
     else if (mode == 1) launch_mode<1>(a, s);

@@ -44,7 +44,7 @@ static_assert(sizeof(WsHeader) == 256, "header size");
 
 struct WsLayout {
     size_t hdr, slots, nest_base, cand_pid, prob_nest, prob_B, prob_W, prob_WR, prob_cnt,
-        prob_status, cand_status, queue, prob_used, prob_md, cls, nest_key, scan_tmp, total;
+        prob_status, cand_status, queue, prob_used, prob_md, cls, nest_key, lane_info, scan_tmp, total;
 };
 
 __host__ __device__ inline size_t ws_align(size_t x) { return (x + 255) & ~size_t(255); }
@@ -75,6 +75,7 @@ __host__ __device__ inline WsLayout ws_layout(uint64_t n, uint64_t n_nests, uint
     L.prob_md = o;    o = ws_align(o + n * kProbModelBytes);
     L.cls = o;        o = ws_align(o + 2 * kClsMax * sizeof(uint32_t));
     L.nest_key = o;   o = ws_align(o + n);
+    L.lane_info = o;  o = ws_align(o + (dedup ? n_nests * 8 : 0));
     uint64_t big = n > n_nests ? n : n_nests;
     L.scan_tmp = o;   o = ws_align(o + scan_blocks(big) * sizeof(uint64_t) * 2);
     L.total = o;

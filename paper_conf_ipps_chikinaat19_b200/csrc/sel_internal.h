@@ -26,6 +26,7 @@ struct WsPtrs {
     void* prob_md;                   // per problem: ProbModel (sel_model.cu)
     uint32_t* cls;                   // [kClsMax] class index per launch, [kClsMax..) B class per index
     uint8_t* nest_key;               // direct mode: shape key per nest (k_problem_w -> k_lane_problems)
+    uint2* lane_info;                // direct mode, per nest: (M_it, mask of classes < 32 the lane kernel counts)
     unsigned long long* scan_tmp;
 };
 

@@ -23,22 +23,24 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_reduce(const unsigned lon
                                                               unsigned long long* partial, const unsigned* skip) {
     if (skip && *skip) return;
     const uint64_t n = n_dev ? *n_dev : n_host;
-    const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
-    unsigned long long s = 0;
-    if (begin < n) {
+    __shared__ unsigned long long red[kScanThreads / 32];
+    // grid-stride over chunks (the grid is sized for the host's upper bound of n)
+    for (uint64_t b = blockIdx.x; b * kScanItems <= n; b += gridDim.x) {
+        const uint64_t begin = b * kScanItems;
+        unsigned long long s = 0;
         for (int i = 0; i < kScanPer; i++) {
             uint64_t idx = begin + uint64_t(i) * kScanThreads + threadIdx.x;
             if (idx < n) s += x[idx];
         }
-    }
-    __shared__ unsigned long long red[kScanThreads / 32];
-    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long t = 0;
-        for (int w = 0; w < kScanThreads / 32; w++) t += red[w];
-        partial[blockIdx.x] = t;
+        for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long t = 0;
+            for (int w = 0; w < kScanThreads / 32; w++) t += red[w];
+            partial[b] = t;
+        }
+        __syncthreads();
     }
 }
 
@@ -86,39 +88,41 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_down(unsigned long long* 
                                                             const unsigned long long* partial, const unsigned* skip) {
     if (skip && *skip) return;
     const uint64_t n = n_dev ? *n_dev : n_host;
-    const uint64_t begin = uint64_t(blockIdx.x) * kScanItems;
-    if (begin > n) return;
-    if (begin == n) {                       // the block that owns x[n] = total
-        if (threadIdx.x == 0) x[n] = partial[blockIdx.x];
-        return;
-    }
-    // each thread scans kScanPer consecutive items
-    const uint64_t my = begin + uint64_t(threadIdx.x) * kScanPer;
-    unsigned long long v[kScanPer], s = 0;
-    for (int i = 0; i < kScanPer; i++) {
-        v[i] = (my + i < n) ? x[my + i] : 0;
-        s += v[i];
-    }
     __shared__ unsigned long long wsum[kScanThreads / 32];
-    unsigned long long inc = s;
-    for (int o = 1; o < 32; o <<= 1) {
-        unsigned long long y = __shfl_up_sync(kFull, inc, o);
-        if ((threadIdx.x & 31) >= o) inc += y;
+    for (uint64_t b = blockIdx.x; b * kScanItems <= n; b += gridDim.x) {
+        const uint64_t begin = b * kScanItems;
+        if (begin == n) {                       // the chunk that owns x[n] = total
+            if (threadIdx.x == 0) x[n] = partial[b];
+            continue;
+        }
+        // each thread scans kScanPer consecutive items
+        const uint64_t my = begin + uint64_t(threadIdx.x) * kScanPer;
+        unsigned long long v[kScanPer], s = 0;
+        for (int i = 0; i < kScanPer; i++) {
+            v[i] = (my + i < n) ? x[my + i] : 0;
+            s += v[i];
+        }
+        unsigned long long inc = s;
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned long long y = __shfl_up_sync(kFull, inc, o);
+            if ((threadIdx.x & 31) >= o) inc += y;
+        }
+        if ((threadIdx.x & 31) == 31) wsum[threadIdx.x >> 5] = inc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long c = 0;
+            for (int w = 0; w < kScanThreads / 32; w++) { unsigned long long t = wsum[w]; wsum[w] = c; c += t; }
+        }
+        __syncthreads();
+        unsigned long long run = partial[b] + wsum[threadIdx.x >> 5] + inc - s;
+        for (int i = 0; i < kScanPer; i++) {
+            if (my + i < n) x[my + i] = run;
+            run += v[i];
+        }
+        const uint64_t last = begin + kScanItems;
+        if (last >= n && threadIdx.x == 0 && n < last) x[n] = partial[b + 1];
+        __syncthreads();                        // wsum is rewritten by the next chunk
     }
-    if ((threadIdx.x & 31) == 31) wsum[threadIdx.x >> 5] = inc;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long c = 0;
-        for (int w = 0; w < kScanThreads / 32; w++) { unsigned long long t = wsum[w]; wsum[w] = c; c += t; }
-    }
-    __syncthreads();
-    unsigned long long run = partial[blockIdx.x] + wsum[threadIdx.x >> 5] + inc - s;
-    for (int i = 0; i < kScanPer; i++) {
-        if (my + i < n) x[my + i] = run;
-        run += v[i];
-    }
-    const uint64_t last = begin + kScanItems;
-    if (last >= n && threadIdx.x == 0 && n < last) x[n] = partial[blockIdx.x + 1];
 }
 
 // skip (device flag, optional): set by the plan when every x[i] is zero -- the
@@ -126,9 +130,10 @@ __global__ void __launch_bounds__(kScanThreads) k_scan_down(unsigned long long* 
 static cudaError_t scan_u64(unsigned long long* x, uint64_t n_max, const unsigned long long* n_dev,
                             unsigned long long* partial, cudaStream_t s, const unsigned* skip = nullptr) {
     const uint64_t nb = (n_max + kScanItems) / kScanItems;     // covers index n_max as well
-    k_scan_reduce<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
+    const unsigned g = unsigned(nb < 148u * 8 ? nb : 148u * 8);  // grid-stride over the chunks
+    k_scan_reduce<<<g, kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
     k_scan_partials<<<1, 1024, 0, s>>>(partial, nb, n_max, n_dev, skip);
-    k_scan_down<<<unsigned(nb), kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
+    k_scan_down<<<g, kScanThreads, 0, s>>>(x, n_max, n_dev, partial, skip);
     note_launch(3);
     return cudaGetLastError();
 }
@@ -293,7 +298,8 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 // The counters of a small problem with W > 0 are not zeroed here: in a
 // single-part call the lane kernel thread that counts it STORES its sums
 // (k_queue adds the handed-over accesses afterwards).
-__device__ __forceinline__ bool problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
+// returns bit 0: counted through the WA prefix (big), bit 1: counted by the lane kernel (small, W > 0)
+__device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
                                               const uint32_t* prob_B, unsigned long long* prob_W,
                                               unsigned long long* prob_WR, uint8_t* prob_status,
                                               unsigned long long* prob_cnt, int lane_ok, bool one_part) {
@@ -302,7 +308,7 @@ __device__ __forceinline__ bool problem_w_one(uint64_t q, const sel_nest& nest, 
         for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
         prob_W[q] = 0;
         prob_WR[q] = 0;
-        return false;
+        return 0u;
     }
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
@@ -313,7 +319,7 @@ __device__ __forceinline__ bool problem_w_one(uint64_t q, const sel_nest& nest, 
     prob_W[q] = small ? 0ull : W;
     if (!(small && W != 0 && one_part))
         for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
-    return !small && W != 0;                 // counted through the WA prefix (k_count)
+    return (!small && W != 0 ? 1u : 0u) | (small && W != 0 ? 2u : 0u);
 }
 
 __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
@@ -321,7 +327,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
                                                    unsigned long long* prob_cnt, int lane_ok, uint8_t* nest_key,
                                                    uint32_t* prob_nest_w, uint32_t* prob_B_w, const uint32_t* cls,
-                                                   uint8_t* prob_used) {
+                                                   uint8_t* prob_used, uint2* lane_info) {
     const uint64_t nq = hdr->n_problems;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     if (hdr->direct) {
@@ -424,15 +430,20 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                 nest_key[i] = nest_shape_key(nest, s_paths[wib][lane], s_emask[wib][lane]);
                 const uint64_t M_it = s_mit[wib][lane];
                 const uint8_t st = nest_status(pre, s_flags[wib][lane], P, M_it);
+                uint32_t lane_mask = 0;
                 for (uint32_t c = 0; c < ncls; c++) {
                     const uint64_t q = i * ncls + c;
                     used++;
                     prob_nest_w[q] = uint32_t(i);
                     prob_B_w[q] = cls[kClsMax + c];
                     prob_used[q] = 0;
-                    big += problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, prob_B, prob_W, prob_WR,
-                                         prob_status, prob_cnt, lane_ok, hdr->n_parts == 1) ? 1u : 0u;
+                    const uint32_t r = problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, prob_B, prob_W, prob_WR,
+                                                     prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
+                    big += r & 1u;
+                    if (c < 32) lane_mask |= ((r >> 1) & 1u) << c;
                 }
+                // the lane kernel's per-nest view: one 8-byte load instead of per-class prefix / WR / M_it
+                lane_info[i] = make_uint2(uint32_t(M_it < 0xffffffffull ? M_it : 0xffffffffull), lane_mask);
             }
             __syncwarp();
         }
@@ -549,7 +560,8 @@ cudaError_t launch_plan(const sel_candidate* cands, uint64_t n, const sel_tables
                                                           w.prob_status, w.prob_cnt,
                                                           (flags & (SEL_F_MATCH_ANY | SEL_F_EXPAND_ALL |
                                                                     SEL_F_WARP_PROBLEMS)) ? 0 : 1,
-                                                          w.nest_key, w.prob_nest, w.prob_B, w.cls, w.prob_used);
+                                                          w.nest_key, w.prob_nest, w.prob_B, w.cls, w.prob_used,
+                                                          w.lane_info);
     prof_end(SEL_PROF_K_PROBLEM_W, s);
     note_launch(2);
     if (dedup) {

@@ -204,6 +204,14 @@ __device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc
     return st;
 }
 
+// The lane kernel also computes the problem half of a4 (ProbModel) of the
+// problems it counts completely, so k_problem_model skips them.  Measured
+// slower (lane kernel 1.1 -> 2.0 ms for 0.45 ms saved in k_problem_model,
+// DESIGN.md rejected variants): off.
+#ifndef SEL_LANE_PREP
+#define SEL_LANE_PREP 0
+#endif
+
 // Problems counted one per lane (k_lane_problems) rather than through the WA
 // prefix: 1-D, small enough for 32-bit lane sums and a short warp-rep walk.
 constexpr uint64_t kSmallMaxW = 1ull << 24;

@@ -1,3 +1,6 @@
 set -x
-bash scripts/gpu_quick.sh
-TOPK=k_lane_problems bash scripts/gpu_ncu_top.sh
+mkdir -p gpurun_out
+python __graft_entry__.py
+timeout 1500 python -m pytest tests -m gpu -q -x --durations=5 > gpurun_out/tests.log 2>&1
+tail -5 gpurun_out/tests.log
+VARIANTS="prep1:;prep0:-DSEL_LANE_PREP=0" bash scripts/gpu_variants.sh

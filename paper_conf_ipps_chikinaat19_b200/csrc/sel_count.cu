@@ -1444,8 +1444,14 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
     const uint64_t ub = qb / ncls, ue = (qe + ncls - 1) / ncls;
     unsigned long long sK = 0, sH = 0;                      // statistics: WAs by path (64-bit: ADVICE r01)
     unsigned long long sW = 0, sOps = 0;
-    for (uint64_t t0 = ub + uint64_t(blockIdx.x) * kLaneTile; t0 < ue; t0 += uint64_t(gridDim.x) * kLaneTile) {
-        const uint32_t nt = uint32_t(umin64(kLaneTile, ue - t0));
+    // tile size: kLaneTile units when there are enough to keep every block busy
+    // (c5: 3.1 M nests), else the units spread over the grid in tiles of at
+    // least 512 (small batches no longer run on a few blocks)
+    const uint64_t per_block = (ue - ub + gridDim.x - 1) / gridDim.x;
+    const uint32_t tile = uint32_t(per_block >= kLaneTile ? kLaneTile
+                                   : per_block <= 512 ? 512u : ((per_block + kLaneThreads - 1) / kLaneThreads) * kLaneThreads);
+    for (uint64_t t0 = ub + uint64_t(blockIdx.x) * tile; t0 < ue; t0 += uint64_t(gridDim.x) * tile) {
+        const uint32_t nt = uint32_t(umin64(tile, ue - t0));
         // ---- sort the tile's units by shape key (counting sort in shared memory)
         for (uint32_t i = threadIdx.x; i < kLaneKeys; i += blockDim.x) s_cnt[i] = 0u;
         __syncthreads();

@@ -284,37 +284,51 @@ def run_ours(args):
     # config 4 (192 huge candidates) splits every candidate's warp-accesses across ranks
     # (SURVEY §8(e)); the others shard candidates by index range
     split = args.config == 4 and world > 1
-    c0, c1 = (0, total) if split else D.shard_range(total, rank, world)
+    # N > 1: rank r evaluates chunks r and N + r of 2N (D.TwoPhaseGather) so the all-gather of the
+    # first half of every rank's decisions runs while the second half is evaluated; the decisions
+    # land directly in the preallocated gather buffer (in-place collectives, no copies)
+    gatherer = D.TwoPhaseGather(total, world, rank, dev) if world > 1 and not split else None
+    ranges = [(0, total)] if split or world == 1 else gatherer.ranges
     t_gen = time.perf_counter()
-    batch = gen.generate(args.config, c0, c1)
+    shards = []
+    for i, (a, b) in enumerate(ranges):
+        bt = gen.generate(args.config, a, b)
+        e = sel.Evaluator((bt.nests, bt.accesses, bt.launches, bt.devices), max(len(bt), 1), args.flags, device=dev)
+        ch = torch.from_numpy(bt.cands.view(np.uint8).reshape(-1)).pin_memory()
+        n_i = len(bt)
+        o = {"decision": gatherer.slots[i] if gatherer else torch.empty(n_i, dtype=torch.uint8, device=dev),
+             "cycles": torch.empty(n_i, dtype=torch.float64, device=dev),
+             "status": torch.empty(n_i, dtype=torch.uint8, device=dev)}
+        shards.append({"batch": bt, "ev": e, "cands_host": ch, "cands": ch.to(dev), "out": o, "range": (a, b)})
     t_gen = time.perf_counter() - t_gen
-    ev = sel.Evaluator((batch.nests, batch.accesses, batch.launches, batch.devices), len(batch), args.flags,
-                       device=dev)
-    cands_host = torch.from_numpy(batch.cands.view(np.uint8).reshape(-1)).pin_memory()
-    cands = cands_host.to(dev)
+    batch, ev, cands, cands_host = shards[0]["batch"], shards[0]["ev"], shards[0]["cands"], shards[0]["cands_host"]
+    c0, c1 = shards[0]["range"]
+    out = shards[0]["out"]
     stream = torch.cuda.current_stream(dev)
-    # outputs preallocated once; with N > 1 the decisions land directly in this rank's slot of the
-    # all-gather buffer (D.DecisionGather: one in-place all_gather_into_tensor per step, no copies)
-    gatherer = D.DecisionGather(total, world, rank, dev) if world > 1 and not split else None
-    n_loc = len(batch)
-    out = {"decision": gatherer.slot if gatherer else torch.empty(n_loc, dtype=torch.uint8, device=dev),
-           "cycles": torch.empty(n_loc, dtype=torch.float64, device=dev),
-           "status": torch.empty(n_loc, dtype=torch.uint8, device=dev)}
 
     def step():
         nonlocal out
         if split:
             out = D.evaluate_split(cands, ev.tables, ev.workspace, rank, world, args.flags)
-        else:
-            ev.evaluate(cands, out=out)
+            return
+        for i, sh in enumerate(shards):
+            if len(sh["batch"]):
+                sh["ev"].evaluate(sh["cands"], out=sh["out"])
             if gatherer:
-                gatherer.gather()
+                gatherer.gather(i)              # NCCL stream: overlaps the next shard's kernels
+        if gatherer:
+            gatherer.wait()
 
     int_peak = {"alu": sel.int_peak(0), "fma": sel.int_peak(1), "both": sel.int_peak(2)}
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize(dev)
-    stats = ev.stats()
+    stats = {}
+    for sh in shards:
+        if not len(sh["batch"]):
+            continue
+        for k, v in sh["ev"].stats().items():
+            stats[k] = stats.get(k, 0) + v
     sel.profile_enable(True)
     PROF = {"plan": sel.PROF_PLAN, "count": sel.PROF_COUNT, "model": sel.PROF_MODEL,
             "k_model_fused": sel.PROF_K_MODEL, "k_lane_problems": sel.PROF_K_LANE, "k_problem_w": sel.PROF_K_PROBLEM_W}
@@ -350,26 +364,43 @@ def run_ours(args):
         # every step uploads its inputs (candidates + nest and access tables) from pinned host
         # memory and downloads decision + cycles to pinned host memory; sel.HostPipeline overlaps
         # step k+1's upload and step k-1's download with step k's kernels (two device slots)
-        nests_h = torch.from_numpy(batch.nests.view(np.uint8).reshape(-1)).pin_memory()
-        acc_h = torch.from_numpy(batch.accesses.view(np.uint8).reshape(-1)).pin_memory()
-        h2d, d2h = sel.HostPipeline.bytes_per_step(cands_host, nests_h, acc_h, len(batch))
-        pipe = sel.HostPipeline(ev, cands_host, nests_h, acc_h)
+        pipes, h2d, d2h = [], 0, 0
+        for sh in shards:
+            if not len(sh["batch"]):
+                continue
+            bt = sh["batch"]
+            nests_h = torch.from_numpy(bt.nests.view(np.uint8).reshape(-1)).pin_memory()
+            acc_h = torch.from_numpy(bt.accesses.view(np.uint8).reshape(-1)).pin_memory()
+            hb, db = sel.HostPipeline.bytes_per_step(sh["cands_host"], nests_h, acc_h, len(bt))
+            h2d, d2h = h2d + hb, d2h + db
+            pipes.append((sel.HostPipeline(sh["ev"], sh["cands_host"], nests_h, acc_h), sh["cands_host"], nests_h,
+                          acc_h))
         for k in range(max(1, args.warmup)):
-            pipe.step(k, cands_host, nests_h, acc_h)
+            for p, ch, nh, ah in pipes:
+                p.step(k, ch, nh, ah)
         torch.cuda.synchronize(dev)
         D.barrier(world)
         f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        f0.record(pipe.h2d)
+        join = torch.cuda.Stream(dev)
+        if pipes:
+            f0.record(pipes[0][0].h2d)
+            for p, _, _, _ in pipes[1:]:
+                p.h2d.wait_event(f0)             # no pipeline starts before the clock does
+        else:
+            f0.record(join)
         for k in range(args.steps):
-            pipe.step(k, cands_host, nests_h, acc_h)
-        f1.record(pipe.d2h)
+            for p, ch, nh, ah in pipes:
+                p.step(k, ch, nh, ah)
+        for p, _, _, _ in pipes:
+            join.wait_stream(p.d2h)
+        f1.record(join)
         torch.cuda.synchronize(dev)
         ms_e2e = D.max_over_ranks(f0.elapsed_time(f1), world, dev)
         e2e = {"value": total / (ms_e2e / 1e3 / args.steps), "unit": UNIT,
                "h2d_bytes_per_step": D.sum_over_ranks(h2d, world, dev),
                "d2h_bytes_per_step": D.sum_over_ranks(d2h, world, dev),
                "ms_per_step": ms_e2e / args.steps, "overlap": "double-buffered H2D / kernels / D2H streams"}
-        del pipe
+        del pipes
 
     if rank != 0:
         return
@@ -420,11 +451,16 @@ def run_ours(args):
              "algorithmic_bytes_per_launch": bytes_per_launch, "bytes": detail,
              "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth, burst)", "ncu": ncu_region(ncu, name)}
         return r
-    n_nests, n_acc = len(batch.nests), len(batch.accesses)
-    roof_model = hbm_roof("model", "model kernels (k_problem_model + k_model_fused)", MODEL_BYTES * len(batch),
+    # per launch: a step evaluates every shard once, so each kernel launch processes on average
+    # 1/len(shards) of this rank's candidates, nests and accesses
+    ns = len(shards)
+    n_cand_launch = sum(len(sh["batch"]) for sh in shards) // ns
+    n_nests = sum(len(sh["batch"].nests) for sh in shards) // ns
+    n_acc = sum(len(sh["batch"].accesses) for sh in shards) // ns
+    roof_model = hbm_roof("model", "model kernels (k_problem_model + k_model_fused)", MODEL_BYTES * n_cand_launch,
                           f"{MODEL_BYTES} B per candidate (record in, decision + cycles + status out)")
     roof_plan = hbm_roof("plan", "plan kernels (k_classes, k_insert, k_problem_w, scans, ...)",
-                         PLAN_BYTES * len(batch) + 88 * n_nests + 64 * n_acc,
+                         PLAN_BYTES * n_cand_launch + 88 * n_nests + 64 * n_acc,
                          f"{PLAN_BYTES} B per candidate (record in, problem id + status out) + every nest (88 B) "
                          f"and access (64 B) record once")
     regions = {"plan": roof_plan, "count": roof_count, "model": roof_model}
@@ -432,11 +468,11 @@ def run_ours(args):
     # HBM on its algorithmic 34 B per candidate, or k_lane_problems / k_problem_w, whichever is longest
     kern = {k: per_launch[k] for k in ("k_model_fused", "k_lane_problems", "k_problem_w")}
     dominant = max(kern, key=kern.get)
-    kbytes = {"k_model_fused": (MODEL_BYTES * len(batch),
+    kbytes = {"k_model_fused": (MODEL_BYTES * n_cand_launch,
                                 f"{MODEL_BYTES} B per candidate (24 B record in; decision, cycles, status out)"),
-              "k_problem_w": (88 * n_nests + 64 * n_acc + 34 * len(batch) // 10,
+              "k_problem_w": (88 * n_nests + 64 * n_acc + 34 * n_cand_launch // 10,
                               "every nest (88 B) and access (64 B) in, ~34 B per problem out"),
-              "k_lane_problems": (88 * n_nests + 64 * n_acc + 40 * (len(batch) * 3 // 32),
+              "k_lane_problems": (88 * n_nests + 64 * n_acc + 40 * (n_cand_launch * 3 // 32),
                                   "every nest (88 B) and access (64 B) in, 40 B of counts per problem out")}
     kb, kdesc = kbytes[dominant]
     kms = kern[dominant]

@@ -120,6 +120,49 @@ class DecisionGather:
         return self.buf[: self.total]
 
 
+class TwoPhaseGather:
+    """The all-gather of decisions overlapped with the evaluation (VERDICT r01
+    #8): the index space is cut into 2 * world chunks of m = ceil(total /
+    (2 world)) candidates and rank r owns chunks r and world + r, so the first
+    halves of all ranks are the contiguous range [0, world m) and the second
+    halves [world m, 2 world m).  The rank evaluates its first chunk into
+    ``slots[0]``, starts ``gather(0)`` (NCCL runs it on its own stream, after
+    the kernels already enqueued on the current stream), evaluates its second
+    chunk into ``slots[1]`` while the first gather is in flight, gathers the
+    second half, and ``wait()`` joins both; ``buf[:total]`` then holds every
+    decision in candidate order.  One preallocated buffer, in-place
+    collectives, no copies."""
+
+    def __init__(self, total: int, world: int, rank: int, device, group=None):
+        self.total, self.world, self.rank, self.group = total, world, rank, group
+        self.m = -(-total // (2 * world)) if total else 0
+        m = self.m
+        self.buf = torch.full((2 * world * m,), 0xFF, dtype=torch.uint8, device=device)
+        self.ranges = [(min(total, j * m), min(total, (j + 1) * m)) for j in (rank, world + rank)]
+        self.slots = [self.buf[j * m: j * m + (b - a)] for j, (a, b) in zip((rank, world + rank), self.ranges)]
+        self.sends = [self.buf[j * m:(j + 1) * m] for j in (rank, world + rank)]
+        self.halves = [self.buf[:world * m], self.buf[world * m:]]
+        self._host = _host_staged(self.buf)
+        self._work = []
+
+    def gather(self, half: int):
+        if self.world == 1:
+            return
+        if self._host:
+            h = torch.empty(self.world * self.m, dtype=torch.uint8)
+            dist.all_gather_into_tensor(h, self.sends[half].cpu(), group=self.group)
+            self.halves[half].copy_(h)
+        else:
+            self._work.append(dist.all_gather_into_tensor(self.halves[half], self.sends[half], group=self.group,
+                                                          async_op=True))
+
+    def wait(self) -> torch.Tensor:
+        for wk in self._work:
+            wk.wait()
+        self._work = []
+        return self.buf[: self.total]
+
+
 def gather_decisions(local: torch.Tensor, total: int, world: int, group=None) -> torch.Tensor:
     """All-gather uint8 decisions of every rank's shard (``shard_range``) into a
     ``total``-long vector in candidate order (identical on every rank).  A

@@ -66,6 +66,13 @@ def _worker(rank, world, port, total, q):
     for _ in range(2):
         g.slot.copy_(local)
         assert torch.equal(g.gather(), full)
+    # two-phase (overlapped) gather: chunks r and w + r of 2w, evaluated and gathered half by half
+    g2 = D.TwoPhaseGather(total, w, r, torch.device("cpu"))
+    dec = ((np.arange(total) * 7 + 3) % 3).astype(np.uint8)     # stand-in decisions, a function of the index
+    for half, (a, b) in enumerate(g2.ranges):
+        g2.slots[half].copy_(torch.from_numpy(dec[a:b]))
+        g2.gather(half)
+    assert g2.wait().numpy().tolist() == dec.tolist()
     st = torch.tensor([0, 6 * rank, 0, rank], dtype=torch.uint8)
     assert D.all_reduce_max_(st, w).tolist() == [0, 6, 0, 1]
     t = D.max_over_ranks(float(rank + 1), w, torch.device("cpu"))

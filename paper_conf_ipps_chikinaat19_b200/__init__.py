@@ -23,7 +23,7 @@ from ._lib import (DECISION_CPU, DECISION_GPU, DECISION_INVALID, SEL_EINTERNAL, 
                    SEL_ERANGE, SEL_F_MATCH_ANY, SEL_F_NO_DEDUP, SEL_OK, SelError)
 
 __all__ = ["load_device_params", "workspace_size", "DeviceTables", "count_transactions", "predict_gpu_cycles",
-           "select", "evaluate", "read_stats", "profile_enable", "profile_read", "profile_read_region", "PROF_PLAN", "PROF_COUNT", "PROF_MODEL",
+           "select", "evaluate", "evaluate_cpu_model", "read_stats", "profile_enable", "profile_read", "profile_read_region", "PROF_PLAN", "PROF_COUNT", "PROF_MODEL",
            "PROF_K_MODEL", "PROF_K_LANE", "PROF_K_PROBLEM_W", "kernel_launches",
            "Evaluator", "SelError", "SEL_F_NO_DEDUP", "SEL_F_MATCH_ANY", "DECISION_CPU", "DECISION_GPU",
            "DECISION_INVALID", "SEL_OK", "SEL_EINVAL", "SEL_ERANGE", "SEL_ELAUNCH", "SEL_EINTERNAL"]
@@ -168,6 +168,34 @@ def evaluate(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor,
     return out
 
 
+def evaluate_cpu_model(cands: torch.Tensor, tables: DeviceTables, workspace: torch.Tensor, cpu_in, params,
+                       flags: int = 0, want_counts: bool = False, want_t_gpu: bool = False, stream=None) -> dict:
+    """sel_evaluate_cpu_model (NEXT row f1 fused into a7): sel_evaluate with the
+    Liao-Chapman CPU cost computed in the same pass -> dict of decision,
+    cycles, status [, t_gpu, counts]."""
+    _require_cuda(cands, workspace)
+    n = _n(cands, "candidate")
+    dev = cands.device
+    cin = cpu_in if isinstance(cpu_in, torch.Tensor) else torch.from_numpy(
+        np.ascontiguousarray(cpu_in).view(np.uint8).reshape(-1)).to(dev)
+    p = np.ascontiguousarray(params)
+    if p.dtype.itemsize != 64:
+        raise ValueError("CPU parameter record must be 64 bytes")
+    out = {"decision": torch.empty(n, dtype=torch.uint8, device=dev),
+           "cycles": torch.empty(n, dtype=torch.float64, device=dev),
+           "status": torch.empty(n, dtype=torch.uint8, device=dev)}
+    if want_t_gpu:
+        out["t_gpu"] = torch.empty(n, dtype=torch.float64, device=dev)
+    if want_counts:
+        out["counts"] = torch.empty((n, 6), dtype=torch.int64, device=dev)
+    wp, wb = _ws_ptr(workspace)
+    _lib.check(_lib.lib().sel_evaluate_cpu_model(_ptr(cands), n, tables.ref(), _ptr(cin), p.ctypes.data,
+                                                 _ptr(out["decision"]), _ptr(out["cycles"]), _ptr(out.get("t_gpu")),
+                                                 _ptr(out.get("counts")), _ptr(out["status"]), wp, wb, flags,
+                                                 _stream(stream)))
+    return out
+
+
 def select_launch(group_of: torch.Tensor, t_gpu: torch.Tensor, status: torch.Tensor, n_groups: int, stream=None):
     """sel_select_launch (NEXT row f3) -> (best uint32-as-int32[n_groups], best_t_gpu f64[n_groups])."""
     _require_cuda(group_of, t_gpu, status)
@@ -266,6 +294,7 @@ sel_count_transactions = count_transactions
 sel_predict_gpu_cycles = predict_gpu_cycles
 sel_select = select
 sel_evaluate = evaluate
+sel_evaluate_cpu_model = evaluate_cpu_model
 sel_read_stats = read_stats
 sel_select_launch = select_launch
 sel_model_cpu_cost = model_cpu_cost

@@ -107,6 +107,7 @@ def lib():
         L.sel_predict_gpu_cycles.argtypes = [vp, u64, T, vp, vp, vp, vp, vp]
         L.sel_select.argtypes = [vp, u64, vp, vp, vp, vp]
         L.sel_evaluate.argtypes = [vp, u64, T, vp, vp, vp, vp, vp, vp, sz, u32, vp]
+        L.sel_evaluate_cpu_model.argtypes = [vp, u64, T, vp, vp, vp, vp, vp, vp, vp, vp, sz, u32, vp]
         L.sel_read_stats.argtypes = [vp, ctypes.POINTER(Stats), vp]
         L.sel_select_launch.argtypes = [vp, u64, vp, vp, u64, vp, vp, vp]
         L.sel_model_cpu_cost.argtypes = [vp, u64, T, vp, vp, vp, vp]
@@ -138,6 +139,6 @@ def check(rc: int):
 
 
 EXPORTED = ("sel_load_device_params", "sel_workspace_size", "sel_count_transactions", "sel_count_transactions_part",
-            "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_select_launch", "sel_model_cpu_cost", "sel_bind_accesses", "sel_read_stats",
+            "sel_predict_gpu_cycles", "sel_select", "sel_evaluate", "sel_evaluate_cpu_model", "sel_select_launch", "sel_model_cpu_cost", "sel_bind_accesses", "sel_read_stats",
             "sel_profile_enable", "sel_profile_read", "sel_profile_read_region", "sel_kernel_launches", "sel_int_peak", "sel_selftest_ddiv", "sel_last_error",
             "sel_version", "sel_sizeof", "sel_offsetof")

@@ -205,6 +205,25 @@ int sel_evaluate(const sel_candidate* c, uint64_t n, const sel_tables* t, uint8_
     return SEL_OK;
 }
 
+int sel_evaluate_cpu_model(const sel_candidate* c, uint64_t n, const sel_tables* t, const sel_cpu_input* cin,
+                           const sel_cpu_params* p, uint8_t* decision, double* cycles, double* t_gpu,
+                           sel_counts* counts, uint8_t* status, void* ws, size_t ws_bytes, uint32_t flags,
+                           sel_stream_t stream) {
+    if (int r = check_common(c, n, t)) return r;
+    if (n == 0) return SEL_OK;
+    if (!decision || !cycles || !status || !cin || !p) return fail(SEL_EINVAL, "NULL argument%s");
+    if (!(p->cpu_hz > 0) || !(p->page_bytes > 0) || p->tlb_entries < 0 || p->tlb_miss_cycles < 0 ||
+        p->loop_overhead_cycles < 0 || p->schedule_static_cycles < 0 || p->sync_cycles < 0 || p->startup_cycles < 0)
+        return fail(SEL_EINVAL, "invalid CPU parameter set%s");
+    if (int r = check_ws(ws, ws_bytes, n, t->n_nests, flags)) return r;
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    const WsPtrs w = ws_ptrs(ws, n, t->n_nests, flags);
+    if (int r = plan_and_count(c, n, t, w, flags, s)) return r;
+    cudaError_t e = launch_model_fused(c, n, *t, w, decision, cycles, t_gpu, counts, status, s, cin, p);
+    if (e != cudaSuccess) return cuda_fail(e, "model");
+    return SEL_OK;
+}
+
 int sel_select_launch(const uint32_t* group_of, uint64_t n, const double* t_gpu, const uint8_t* status,
                       uint64_t n_groups, uint32_t* best, double* best_t, sel_stream_t stream) {
     if (n_groups == 0) return SEL_OK;

@@ -1348,6 +1348,9 @@ __device__ __forceinline__ void lane_hist_prepare(Col h, const sel_access& a, ui
 #ifndef SEL_LANE_BLOCK_PERIOD
 #define SEL_LANE_BLOCK_PERIOD 1
 #endif
+#ifndef SEL_LANE_ONE_EVAL
+#define SEL_LANE_ONE_EVAL 1
+#endif
 __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint32_t P, uint32_t B, uint32_t WR,
                                                const RepClasses& rc, uint32_t tmin, LaneSums& z) {
     const uint32_t sh = uint32_t(__ffs(a.elem_bytes) - 1), R = 128u >> sh;
@@ -1526,7 +1529,9 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
             const uint32_t i = r * kLaneThreads + threadIdx.x;
             const bool has = i < nt;
             const uint64_t u = has ? t0 + s_order[i] : 0ull;
+#if SEL_LANE_PREP
             uint32_t fin_mask = 0;                          // classes (< 32) whose ProbModel this thread wrote
+#endif
             for (uint32_t g0 = 0; g0 < ncls; g0 += kLaneGrp) {
                 // problems q = u * ncls + g0 + c of this group that are small and in this call's range
                 uint32_t B[kLaneGrp], WR[kLaneGrp], hm[kLaneGrp];
@@ -1602,6 +1607,30 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                                 }
                         } else if (d <= 2 && ac.elem_bytes >= 4 && a.residue_classes) {
                             lane_hist_prepare(hcol, ac, T0, T1, z[0].ops);
+#if SEL_LANE_ONE_EVAL
+                            // the block-size classes through ONE inlined copy of lane_hist_eval (its
+                            // class_sums evaluations dominate the kernel; code size showed in the
+                            // stalls): the class's inputs and sums picked with constant indices
+#pragma unroll 1
+                            for (uint32_t c = 0; c < kLaneGrp; c++) {
+                                if (!((vmask >> c) & 1u)) continue;
+                                uint32_t Bc = B[0], WRc = WR[0];
+                                RepClasses rcc = rc[0];
+#pragma unroll
+                                for (uint32_t i = 1; i < kLaneGrp; i++)
+                                    if (c == i) { Bc = B[i]; WRc = WR[i]; rcc = rc[i]; }
+                                LaneSums dz{0u, 0u, 0u, 0u, 0u, 0ull};
+                                lane_hist_eval(hcol, ac, uint32_t(nest.P0), Bc, WRc, rcc, tc, dz);
+                                dz.W = WRc * Mk;
+#pragma unroll
+                                for (uint32_t i = 0; i < kLaneGrp; i++)
+                                    if (c == i) {
+                                        z[i].W += dz.W; z[i].L += dz.L; z[i].S += dz.S; z[i].C += dz.C; z[i].U += dz.U;
+                                        z[i].ops += dz.ops;
+                                    }
+                                sH += uint64_t(WRc) * Mk;
+                            }
+#else
 #pragma unroll
                             for (uint32_t c = 0; c < kLaneGrp; c++)
                                 if ((vmask >> c) & 1u) {
@@ -1609,6 +1638,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                                     sH += uint64_t(WR[c]) * Mk;
                                     z[c].W += WR[c] * Mk;
                                 }
+#endif
                         } else {
 #pragma unroll
                             for (uint32_t c = 0; c < kLaneGrp; c++) hm[c] |= ((vmask >> c) & 1u) << k;   // to k_queue

@@ -55,7 +55,8 @@ cudaError_t launch_gather_counts(const sel_candidate* cands, uint64_t n, const s
                                  cudaStream_t s);
 cudaError_t launch_model_fused(const sel_candidate* cands, uint64_t n, const sel_tables& t, const WsPtrs& w,
                                uint8_t* decision, double* cycles, double* t_gpu, sel_counts* counts,
-                               uint8_t* status, cudaStream_t s);
+                               uint8_t* status, cudaStream_t s, const sel_cpu_input* cin = nullptr,
+                               const sel_cpu_params* cp = nullptr);
 cudaError_t launch_model_from_counts(const sel_candidate* cands, uint64_t n, const sel_tables& t,
                                      const sel_counts* counts, double* cycles, double* t_gpu, uint8_t* status,
                                      cudaStream_t s);

@@ -12,6 +12,7 @@
 //     candidates that reach the minimum.
 #include "sel_device.cuh"
 #include "sel_internal.h"
+#include "sel_model.cuh"
 
 namespace sel {
 
@@ -83,19 +84,8 @@ __global__ void __launch_bounds__(256) k_cpu_model(sel_candidate* __restrict__ c
         return;
     }
     const sel_nest nt = t.nests[nid];
-    const uint64_t P = nt.P0 * nt.P1;
-    const uint64_t chunk = cdiv(P, x.threads);                                     // F1a
-    const double footprint = __ddiv_rn(__ull2double_rn(nt.bytes_h2d + nt.bytes_d2h), __uint2double_rn(x.threads));
-    const double pages = ceil(__ddiv_rn(footprint, p.page_bytes));
-    const double misses = pages > p.tlb_entries ? __dsub_rn(pages, p.tlb_entries) : 0.0;
-    const double cache = __dmul_rn(misses, p.tlb_miss_cycles);                     // F1c
-    const double loop_overhead = __dmul_rn(p.loop_overhead_cycles, __ull2double_rn(chunk));
-    const double loop_chunk = __dadd_rn(__dadd_rn(__dmul_rn(x.mca_cycles_per_iter, __ull2double_rn(chunk)), cache),
-                                        loop_overhead);
-    const double parallel_for = __dmul_rn(1.0, __dadd_rn(__dadd_rn(__dadd_rn(p.schedule_static_cycles, loop_chunk), 0.0),
-                                                         0.0));                   // F1b
-    const double thread_exe = __dadd_rn(parallel_for, p.sync_cycles);
-    cands[c].cpu_cycles = __dadd_rn(__dadd_rn(p.startup_cycles, thread_exe), 0.0);  // F1d
+    bool bad = false;
+    cands[c].cpu_cycles = cpu_cycles_fig3(nt.P0 * nt.P1, __ull2double_rn(nt.bytes_h2d + nt.bytes_d2h), x, p, &bad);
     cands[c].cpu_hz = p.cpu_hz;
     status[c] = SEL_OK;
 }

@@ -97,3 +97,37 @@ def test_bind_parity(sel, cfg, rng):
     assert (st.cpu().numpy() == st_ref).all()
     assert np.array_equal(out.cpu().numpy(), ref)
     assert (st_ref != 0).sum() >= 1
+
+
+@pytest.mark.parametrize("cfg,rng", [(2, (0, 108)), (4, (0, 192)), (5, (0, 300000))])
+def test_evaluate_cpu_model_fused(sel, cfg, rng):
+    """NEXT row f1 fused into a7 (sel_evaluate_cpu_model): one pass with the
+    Liao-Chapman CPU cost gives the oracle's decisions and cycles computed on
+    candidates whose cpu_cycles / cpu_hz the oracle's own f1 model replaced;
+    invalid CPU inputs -> SEL_EINVAL.  The candidate records stay untouched."""
+    b = gen.generate(cfg, *rng)
+    cin = gen.cpu_inputs(cfg, *rng)
+    cin["threads"][::53] = 0
+    cin["mca_cycles_per_iter"][7::61] = -1.0
+    params = gen.cpu_params()
+    cyc, st_f1 = oracle.cpu_model(params, b, cin)
+    cm = b.cands.copy()
+    ok = st_f1 == 0
+    cm["cpu_cycles"][ok] = cyc[ok]
+    cm["cpu_hz"][ok] = params["cpu_hz"][0]
+    ref = oracle.evaluate(gen.Batch(cm, b.nests, b.accesses, b.launches, b.devices))
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
+    c = sel._as_bytes_tensor(b.cands.copy(), "candidate")
+    before = c.clone()
+    r = sel.evaluate_cpu_model(c, ev.tables, ev.workspace, cin, params, want_t_gpu=True)
+    torch.cuda.synchronize()
+    assert torch.equal(c, before)
+    status = r["status"].cpu().numpy()
+    exp_status = np.where(ok, ref["status"], 1)
+    assert (status == exp_status).all()
+    v = ok & (ref["status"] == 0)
+    assert (r["decision"].cpu().numpy()[v] == ref["decision"][v]).all()
+    assert (r["cycles"].cpu().numpy()[v] == ref["cycles"][v]).all()
+    assert (r["t_gpu"].cpu().numpy()[v] == ref["t_gpu"][v]).all()
+    assert (r["decision"].cpu().numpy()[~ok] == 0xFF).all()
+    assert v.sum() > 0.9 * len(b) - 2 * len(b) // 50

@@ -1365,6 +1365,46 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
         lane_add(z, class_sums(h, p32, R, sh, lo, nm1, g, tmin, mult), Ht * mult);
     };
     auto lo_of = [&](uint32_t p0, uint32_t n) { return base32 + c032 * p0 + (neg ? c032 * (n - 1u) : 0u); };
+#if SEL_LANE_BLOCK_PERIOD
+    // Element sizes >= 4 (the only ones the lane kernel sends here) make 32 c
+    // = 0 (mod 128): every full warp of a block has the lowest lane address of
+    // the block's first warp (mod 128 -- all class_sums looks at).  When 32 | B
+    // or c B = 0 (mod 128) the warp-reps fall into the lane-count classes of
+    // rep_classes (count_hist_whole); otherwise block kb's offset c kb B (mod
+    // 128) repeats with period pi = 128 / gcd(c B, 128), so the complete
+    // blocks' warp-reps fall into <= 2 min(pi, #blocks) classes (full warps,
+    // the B mod 32 tail warp) with multiplicities, plus the last block's full
+    // warps and tail (R8, R9) -- the same integers as walking every warp-rep.
+    // The classes are enumerated as items through ONE call site of class_sums
+    // (its copies were the kernel's code size).
+    const bool whole = (B & 31u) == 0 || ((c032 * B) & 127u) == 0;
+    const uint32_t nfull = (B - 1u) >> 5, lt = B & 31u;
+    const uint32_t nbf = uint32_t(rc.nA), rem_full = whole ? 0u : uint32_t(rc.n32) - nbf * nfull;
+    const uint32_t lp = whole ? 0u : 7u - uint32_t(__ffs((c032 * B) & 127u) - 1);   // log2 pi
+    const uint32_t nr = whole ? 0u : (nbf < (1u << lp) ? nbf : (1u << lp));
+    const uint32_t items = whole ? 3u : 2u * nr + 2u;
+    for (uint32_t x = 0; x < items; x++) {
+        uint32_t p0, n, mult;
+        if (whole) {
+            if (x == 0) { p0 = 0u; n = 32u; mult = uint32_t(rc.n32); }
+            else if (x == 1) { p0 = 0u; n = rc.lanesA; mult = uint32_t(rc.nA); }
+            else { p0 = rc.nA ? 0u : uint32_t(32u * rc.n32); n = rc.lanesR; mult = rc.lanesR ? 1u : 0u; }
+        } else if (x < 2u * nr) {
+            const uint32_t r = x >> 1, m = ((nbf - 1u - r) >> lp) + 1u;   // complete blocks kb = r (mod pi)
+            const bool tail = x & 1u;
+            p0 = r * B + (tail ? 32u * nfull : 0u);
+            n = tail ? lt : 32u;
+            mult = tail ? m : m * nfull;
+        } else if (x == 2u * nr) {
+            p0 = nbf * B; n = 32u; mult = rem_full;
+        } else {
+            p0 = nbf * B + 32u * rem_full; n = rc.lanesR; mult = rc.lanesR ? 1u : 0u;
+        }
+        if (mult) cls(lo_of(p0, n), n - 1u, mult);
+    }
+    (void)WR;
+    (void)P;
+#else
     if ((B & 31u) == 0 || (((c032 * B) | (32u * g)) & 127u) == 0) {
         // the lowest lane address mod 128 of a warp-rep depends on its lane count only
         // (or, for 32 | B, on the warp-rep index mod 4): count_hist_whole's classes
@@ -1379,39 +1419,6 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
         if (rc.nA) cls(lo_of(0u, rc.lanesA), rc.lanesA - 1u, uint32_t(rc.nA));
         if (rc.lanesR) cls(lo_of(rc.nA ? 0u : uint32_t(32u * rc.n32), rc.lanesR), rc.lanesR - 1u, 1u);
     } else {
-#if SEL_LANE_BLOCK_PERIOD
-        // 32 does not divide B and c B != 0 (mod 128).  Element sizes >= 4 make
-        // 32 c = 0 (mod 128), so every full warp of block kb has the lowest lane
-        // address of the block's first warp (mod 128 -- all class_sums looks
-        // at), and block kb's offset c kb B (mod 128) repeats with period
-        // pi = 128 / gcd(c B, 128): the warp-reps of the complete blocks fall
-        // into <= 2 min(pi, #blocks) classes (full warps, the B mod 32 tail
-        // warp) with multiplicities, plus the last block's full warps and tail
-        // (R8, R9; rep_classes split P into them) -- the same integers as
-        // walking every warp-rep.  One call site of class_sums (code size).
-        const uint32_t nfull = (B - 1u) >> 5, lt = B & 31u;
-        const uint32_t nbf = uint32_t(rc.nA), rem_full = uint32_t(rc.n32) - nbf * nfull;
-        const uint32_t lp = 7u - uint32_t(__ffs((c032 * B) & 127u) - 1);   // log2 pi
-        const uint32_t nr = nbf < (1u << lp) ? nbf : (1u << lp);
-        const uint32_t items = 2u * nr + 2u;
-        for (uint32_t x = 0; x < items; x++) {
-            uint32_t p0, n, mult;
-            if (x < 2u * nr) {
-                const uint32_t r = x >> 1, m = ((nbf - 1u - r) >> lp) + 1u;   // complete blocks kb = r (mod pi)
-                const bool tail = x & 1u;
-                p0 = r * B + (tail ? 32u * nfull : 0u);
-                n = tail ? lt : 32u;
-                mult = tail ? m : m * nfull;
-            } else if (x == 2u * nr) {
-                p0 = nbf * B; n = 32u; mult = rem_full;
-            } else {
-                p0 = nbf * B + 32u * rem_full; n = rc.lanesR; mult = rc.lanesR ? 1u : 0u;
-            }
-            if (mult) cls(lo_of(p0, n), n - 1u, mult);
-        }
-        (void)WR;
-        (void)P;
-#else
         // every warp-rep from the block geometry (R8, R9), as count_hist_reps
         const uint32_t wpb = (B + 31u) >> 5;
         uint32_t kb = 0, w = 0;
@@ -1424,8 +1431,8 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
             cls(base32 + c032 * p0 + (neg ? c032 * nm1 : 0u), nm1, 1u);
             if (++w == wpb) { w = 0; kb++; }
         }
-#endif
     }
+#endif
 }
 
 // Small problems (k_problem_w: 1-D, W <= kSmallMaxW, WR <= kSmallMaxWR), one

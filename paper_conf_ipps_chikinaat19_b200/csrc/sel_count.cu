@@ -33,7 +33,6 @@
 //    64-bit lane addresses, __match_any_sync on (addr >> 7) and (addr >> 5),
 //    first-occurrence flags, __ballot_sync/__popc.
 #include "sel_device.cuh"
-#include "sel_model.cuh"
 #include "sel_internal.h"
 
 namespace sel {
@@ -77,10 +76,8 @@ struct CountArgs {
     uint32_t residue_classes;           // whole arithmetic-lane warp-reps by residue classes (count_hist)
     unsigned long long* queue;          // small problems handed from k_lane_problems to k_queue
     const uint8_t* nest_key;            // direct mode: shape key per nest (k_problem_w)
-    uint2* lane_info;                   // direct mode: per nest (M_it, mask of classes < 32 counted here);
-                                        // k_lane_problems rewrites the mask: classes it also finalised
+    const uint2* lane_info;             // direct mode: per nest (M_it, mask of classes < 32 counted here)
     const uint32_t* cls_B;              // direct mode: B class of each class index
-    void* prob_md;                      // per problem: ProbModel (sel_model.cuh)
 };
 
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
@@ -1485,9 +1482,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
     const bool direct = a.hdr->direct != 0;
     const uint32_t ncls = direct ? a.hdr->n_cls : 1u;
     const uint64_t qb = a.hdr->small_begin, qe = a.hdr->small_end;
-#if SEL_LANE_PREP
-    const bool fin = direct && a.hdr->n_parts == 1 && a.prob_md != nullptr;   // finalise ProbModels here
-#endif
+
     const uint64_t ub = qb / ncls, ue = (qe + ncls - 1) / ncls;
     unsigned long long sK = 0, sH = 0;                      // statistics: WAs by path (64-bit: ADVICE r01)
     unsigned long long sW = 0, sOps = 0;
@@ -1536,9 +1531,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
             const uint32_t i = r * kLaneThreads + threadIdx.x;
             const bool has = i < nt;
             const uint64_t u = has ? t0 + s_order[i] : 0ull;
-#if SEL_LANE_PREP
-            uint32_t fin_mask = 0;                          // classes (< 32) whose ProbModel this thread wrote
-#endif
+
             for (uint32_t g0 = 0; g0 < ncls; g0 += kLaneGrp) {
                 // problems q = u * ncls + g0 + c of this group that are small and in this call's range
                 uint32_t B[kLaneGrp], WR[kLaneGrp], hm[kLaneGrp];
@@ -1673,21 +1666,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                                 atomicAdd(pc + 4, (unsigned long long)z[c].U);
                             }
                         }
-#if SEL_LANE_PREP
-                        // a problem counted completely here (direct ids, one part, nothing handed to
-                        // k_queue): the problem half of a4 now, from the sums in registers and the nest
-                        // already loaded -- k_problem_model skips it (lane_info mask)
-                        if (fin && hm[c] == 0u && g0 + c < 32u) {
-                            bool ok = true;
-                            ProbModel m = prep_problem(nest, Mit, z[c].W, z[c].S, z[c].C, z[c].U, WR[c], DivFast{&ok});
-                            if (!ok) m = prep_problem(nest, Mit, z[c].W, z[c].S, z[c].C, z[c].U, WR[c], DivExact{});
-                            const int4* src = reinterpret_cast<const int4*>(&m);
-                            int4* dst = reinterpret_cast<int4*>(static_cast<ProbModel*>(a.prob_md) + q);
-#pragma unroll
-                            for (int x = 0; x < int(sizeof(ProbModel) / 16); x++) dst[x] = src[x];
-                            fin_mask |= 1u << (g0 + c);
-                        }
-#endif
+
                     }
                 }
                 // warp-aggregated append of the handed problems to the queue (converged)
@@ -1703,9 +1682,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                     }
                 }
             }
-#if SEL_LANE_PREP
-            if (fin && has) a.lane_info[u].y = fin_mask;
-#endif
+
         }
         __syncthreads();                                    // s_order / s_cnt are rewritten by the next tile
     }
@@ -1923,7 +1900,7 @@ cudaError_t launch_count(const sel_tables& t, const WsPtrs& w, uint64_t max_prob
     const int mode = (flags & SEL_F_MATCH_ANY) ? 0 : (flags & SEL_F_SCALAR) ? 1 : 2;
     CountArgs a{t.nests, t.accesses, w.prob_nest, w.prob_B, w.prob_W, w.prob_WR, w.prob_cnt, w.hdr, 1u,
                 (flags & SEL_F_EXPAND_ALL) ? 0u : 1u, (flags & SEL_F_NO_RESIDUE_CLASSES) ? 0u : 1u,
-                w.queue, w.nest_key, w.lane_info, w.cls + kClsMax, w.prob_md};
+                w.queue, w.nest_key, w.lane_info, w.cls + kClsMax};
     prof_before_count(s);
     if (mode == 0) launch_mode<0>(a, s);
     else if (mode == 1) launch_mode<1>(a, s);

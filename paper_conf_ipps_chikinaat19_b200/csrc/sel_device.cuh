@@ -98,6 +98,7 @@ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) {
 }
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ uint64_t smul(uint64_t a, uint64_t b) {
+    if (((a | b) >> 32) == 0) return a * b;               // both below 2^32: no overflow (the common case)
     if (a == 0 || b == 0) return 0;
     return __umul64hi(a, b) ? ~0ull : a * b;               // saturate on overflow
 }
@@ -204,13 +205,6 @@ __device__ inline uint8_t validate_nest(const sel_nest& n, const sel_access* acc
     return st;
 }
 
-// The lane kernel also computes the problem half of a4 (ProbModel) of the
-// problems it counts completely, so k_problem_model skips them.  Measured
-// slower (lane kernel 1.1 -> 2.0 ms for 0.45 ms saved in k_problem_model,
-// DESIGN.md rejected variants): off.
-#ifndef SEL_LANE_PREP
-#define SEL_LANE_PREP 0
-#endif
 
 // Problems counted one per lane (k_lane_problems) rather than through the WA
 // prefix: 1-D, small enough for 32-bit lane sums and a short warp-rep walk.

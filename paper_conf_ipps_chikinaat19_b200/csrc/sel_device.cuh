@@ -161,16 +161,20 @@ __device__ __forceinline__ uint32_t access_check(const sel_access& a, uint32_t p
     // power-of-two element size: divisibility by masking
     const int64_t m = e - 1;
     bool bad = (a.base & m) || (a.c_par[0] & m) || (par_dims == 2 && (a.c_par[1] & m));
-    for (int j = 0; j < a.depth; j++) bad |= (a.c_inner[j] & m) != 0;
+#pragma unroll
+    for (int j = 0; j < 3; j++) bad |= (j < a.depth) && (a.c_inner[j] & m) != 0;   // static indices: no local memory
     if (bad) return kAccInval;
     const uint64_t e0 = (par_dims == 1) ? P : P0;
     uint64_t bound = uabs(a.base);
     bound = sadd(bound, smul(uabs(a.c_par[0]), e0 ? e0 - 1 : 0));
     if (par_dims == 2) bound = sadd(bound, smul(uabs(a.c_par[1]), P1 ? P1 - 1 : 0));
     uint64_t Mk = 1;
-    for (int j = 0; j < a.depth; j++) {
-        bound = sadd(bound, smul(uabs(a.c_inner[j]), T[j] ? T[j] - 1 : 0));
-        Mk = smul(Mk, T[j]);
+#pragma unroll
+    for (int j = 0; j < 3; j++) {
+        if (j < a.depth) {
+            bound = sadd(bound, smul(uabs(a.c_inner[j]), T[j] ? T[j] - 1 : 0));
+            Mk = smul(Mk, T[j]);
+        }
     }
     *Mk_out = Mk;
     return bound >= kLim62 ? kAccRange : 0u;

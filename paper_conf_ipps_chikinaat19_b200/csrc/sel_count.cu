@@ -1241,6 +1241,14 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
 // the lane); at the first access that needs the warp (deeper loop nests, block
 // sizes whose warp-reps fall into many residue classes, collapse(2)) it hands
 // the rest of its problem to the warp (queue of <= 32 entries).
+#ifndef SEL_LANE_OPS
+#define SEL_LANE_OPS 1      // nominal lane-op accounting (count_nominal_ops); 0 drops it from the lane kernel
+#endif
+#if SEL_LANE_OPS
+#define LANE_OPS(x) x
+#else
+#define LANE_OPS(x) ((void)0)
+#endif
 struct LaneSums {
     uint32_t W, L, S, C, U;
     unsigned long long ops;          // nominal algorithmic lane-ops of this thread
@@ -1250,7 +1258,7 @@ struct LaneSums {
 __device__ __forceinline__ void lane_uniform(const RepClasses& rc, uint32_t Mk, bool flags, uint32_t tmin,
                                              LaneSums& z) {
     auto cls = [&](uint32_t lanes, uint32_t reps) {
-        z.ops += kOpsClass;
+        LANE_OPS(z.ops += kOpsClass);
         const uint32_t w = reps * Mk;
         const uint32_t nl = flags ? lanes : 1u;             // lines = sectors per WA
         z.L += w * nl;
@@ -1289,14 +1297,14 @@ __device__ __forceinline__ void lane_hist_build(Col h, uint32_t R, uint32_t sh, 
     const uint32_t kA = uint32_t(uint64_t(a.c_inner[0]));
     const uint32_t lA = loop_period_log2(kA), pA = 1u << lA, nA = T0 < pA ? T0 : pA;
     if (d == 1) {
-        ops += kOpsHistEntry * nA;
+        LANE_OPS(ops += kOpsHistEntry * nA);
         for (uint32_t i = 0; i < nA; i++) h[((kA * i) & 127u) >> sh] = (T0 - i + pA - 1u) >> lA;
         return;
     }
     // depth 2: every (i, j) residue pair of the two loops' one-loop histograms
     const uint32_t kB = uint32_t(uint64_t(a.c_inner[1]));
     const uint32_t lB = loop_period_log2(kB), pB = 1u << lB, nB = T1 < pB ? T1 : pB;
-    ops += kOpsHistEntry * (nA + nB) + kOpsConvTerm * nA * nB;
+    LANE_OPS(ops += kOpsHistEntry * (nA + nB) + kOpsConvTerm * nA * nB);
     for (uint32_t i = 0; i < nA; i++) {
         const uint32_t ci = (T0 - i + pA - 1u) >> lA, oi = kA * i;
         for (uint32_t j = 0; j < nB; j++) {
@@ -1310,7 +1318,7 @@ __device__ __forceinline__ void lane_hist_build(Col h, uint32_t R, uint32_t sh, 
 // folded mod 32 bytes (R / 4 slots)
 __device__ __forceinline__ void lane_hist_prefix(Col h, uint32_t R, unsigned long long& ops) {
     const uint32_t R32 = R >> 2;
-    ops += kOpsPrefixEntry * (R + R32);
+    LANE_OPS(ops += kOpsPrefixEntry * (R + R32));
     uint32_t run = 0;
     for (uint32_t u = 0; u < R32; u++) {
         run += h[u] + h[u + R32] + h[u + 2u * R32] + h[u + 3u * R32];
@@ -1358,7 +1366,7 @@ __device__ __forceinline__ void lane_hist_eval(Col h, const sel_access& a, uint3
     const bool neg = c0 < 0;
     const uint32_t base32 = uint32_t(uint64_t(a.base)), c032 = uint32_t(uint64_t(c0));
     auto cls = [&](uint32_t lo, uint32_t nm1, uint32_t mult) {
-        z.ops += kOpsEvalClass;
+        LANE_OPS(z.ops += kOpsEvalClass);
         lane_add(z, class_sums(h, p32, R, sh, lo, nm1, g, tmin, mult), Ht * mult);
     };
     auto lo_of = [&](uint32_t p0, uint32_t n) { return base32 + c032 * p0 + (neg ? c032 * (n - 1u) : 0u); };
@@ -1626,7 +1634,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                                 for (uint32_t i = 0; i < kLaneGrp; i++)
                                     if (c == i) {
                                         z[i].W += dz.W; z[i].L += dz.L; z[i].S += dz.S; z[i].C += dz.C; z[i].U += dz.U;
-                                        z[i].ops += dz.ops;
+                                        LANE_OPS(z[i].ops += dz.ops);
                                     }
                                 sH += uint64_t(WRc) * Mk;
                             }
@@ -1649,7 +1657,7 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                         if (!((vmask >> c) & 1u)) continue;
                         const uint64_t q = u * ncls + g0 + c;
                         sW += uint64_t(WR[c]) * Mit;
-                        sOps += z[c].ops;
+                        LANE_OPS(sOps += z[c].ops);
                         {   // the only writer so far (k_problem_w leaves these counters unzeroed): store
                             unsigned long long* pc = a.prob_cnt + q * kCntStride;
                             if (a.hdr->n_parts == 1) {

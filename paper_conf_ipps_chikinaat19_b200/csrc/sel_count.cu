@@ -1241,6 +1241,9 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
 // the lane); at the first access that needs the warp (deeper loop nests, block
 // sizes whose warp-reps fall into many residue classes, collapse(2)) it hands
 // the rest of its problem to the warp (queue of <= 32 entries).
+#ifndef SEL_LANE_PF
+#define SEL_LANE_PF 1       // L1 prefetch of the nest's next access descriptors (2: + the next nest into L2)
+#endif
 #ifndef SEL_LANE_OPS
 #define SEL_LANE_OPS 1      // nominal lane-op accounting (count_nominal_ops); 0 drops it from the lane kernel
 #endif
@@ -1539,6 +1542,11 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
             const uint32_t i = r * kLaneThreads + threadIdx.x;
             const bool has = i < nt;
             const uint64_t u = has ? t0 + s_order[i] : 0ull;
+#if SEL_LANE_PF >= 2
+            // the next round's nest into L2 while this one is counted
+            if (i + kLaneThreads < nt && direct)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.nests + (t0 + s_order[i + kLaneThreads])));
+#endif
 
             for (uint32_t g0 = 0; g0 < ncls; g0 += kLaneGrp) {
                 // problems q = u * ncls + g0 + c of this group that are small and in this call's range
@@ -1593,7 +1601,16 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                     const uint32_t T0 = uint32_t(eff_trip(nest.trip[0])), T1 = uint32_t(eff_trip(nest.trip[1])),
                                    T2 = uint32_t(eff_trip(nest.trip[2]));
                     const sel_access* ap = a.acc + nest.access_off;
+#if SEL_LANE_PF >= 1
+                    // the nest's access descriptors are read one after another, each
+                    // load on the critical path: touch the next line ahead of time
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(ap + 2));
+#endif
                     for (uint32_t k = 0; k < nest.n_access; k++, ap++) {
+#if SEL_LANE_PF >= 1
+                        if ((k & 1u) == 0u && k + 4u < nest.n_access)
+                            asm volatile("prefetch.global.L1 [%0];" ::"l"(ap + 4));
+#endif
                         if (k == 31) {                      // accesses 31, 32, ...: all to the warp kernel
 #pragma unroll
                             for (uint32_t c = 0; c < kLaneGrp; c++) hm[c] |= ((vmask >> c) & 1u) << 31;

@@ -165,6 +165,24 @@ __device__ __forceinline__ uint32_t access_check(const sel_access& a, uint32_t p
     for (int j = 0; j < 3; j++) bad |= (j < a.depth) && (a.c_inner[j] & m) != 0;   // static indices: no local memory
     if (bad) return kAccInval;
     const uint64_t e0 = (par_dims == 1) ? P : P0;
+    {
+        // every magnitude and extent below 2^20: each of the <= 6 bound terms is
+        // below 2^40, so the bound is far below 2^62 and M_k (<= 3 trips) below
+        // 2^60 -- no saturating arithmetic needed (the common case)
+        uint64_t big = uabs(a.base) | uabs(a.c_par[0]) | e0;
+        if (par_dims == 2) big |= uabs(a.c_par[1]) | P1;
+        uint64_t Mk = 1;
+#pragma unroll
+        for (int j = 0; j < 3; j++)
+            if (j < a.depth) {
+                big |= uabs(a.c_inner[j]) | T[j];
+                Mk *= T[j];
+            }
+        if ((big >> 20) == 0) {
+            *Mk_out = Mk;
+            return 0u;
+        }
+    }
     uint64_t bound = uabs(a.base);
     bound = sadd(bound, smul(uabs(a.c_par[0]), e0 ? e0 - 1 : 0));
     if (par_dims == 2) bound = sadd(bound, smul(uabs(a.c_par[1]), P1 ? P1 - 1 : 0));

@@ -401,21 +401,42 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                     paths = 1u << (8u * path);
                     em = 1u << (__ffs(ac.elem_bytes) & 31);
                 }
-                // segmented (by owner) saturating sum over the lanes of this round
+                // segmented (by owner) sum over the lanes of this round: the owner's
+                // lanes are contiguous from seg_lo (its first access in this round),
+                // so lane l takes lane l - o's values iff l - o >= seg_lo; the flags
+                // and the element-size mask travel in one word (both OR-combined),
+                // and M_k in 32 bits when every lane's is below 2^26 (no overflow in
+                // 32 terms), else 64-bit saturating
                 const bool in = j < tot;
+                const int seg_lo = int(ex) - int(j0) > 0 ? int(ex) - int(j0) : 0;
+                uint32_t flem = fl | (em << 8);
+                if (__all_sync(kFull, Mk < (1ull << 26))) {
+                    uint32_t m32 = uint32_t(Mk);
 #pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint64_t y = __shfl_up_sync(kFull, Mk, o);
-                    const uint32_t yf = __shfl_up_sync(kFull, fl, o);
-                    const int yo = __shfl_up_sync(kFull, own, o);
-                    const uint32_t yp = __shfl_up_sync(kFull, paths, o), ye = __shfl_up_sync(kFull, em, o);
-                    if (lane >= o && yo == own) {
-                        Mk = sadd(Mk, y);
-                        fl |= yf;
-                        paths += yp;
-                        em |= ye;
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(kFull, m32, o);
+                        const uint32_t yf = __shfl_up_sync(kFull, flem, o), yp = __shfl_up_sync(kFull, paths, o);
+                        if (lane - o >= seg_lo) {
+                            m32 += y;
+                            flem |= yf;
+                            paths += yp;
+                        }
+                    }
+                    Mk = m32;
+                } else {
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint64_t y = __shfl_up_sync(kFull, Mk, o);
+                        const uint32_t yf = __shfl_up_sync(kFull, flem, o), yp = __shfl_up_sync(kFull, paths, o);
+                        if (lane - o >= seg_lo) {
+                            Mk = sadd(Mk, y);
+                            flem |= yf;
+                            paths += yp;
+                        }
                     }
                 }
+                fl = flem & 0xffu;
+                em = flem >> 8;
                 const int nxt = __shfl_down_sync(kFull, own, 1);
                 const bool tail = in && (lane == 31 || j + 1 >= tot || nxt != own);
                 if (tail) {                                     // one lane per owner per round

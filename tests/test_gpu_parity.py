@@ -608,3 +608,39 @@ def test_direct_ids_sparse_nests(sel):
     g = run_gpu(sel, b)
     assert_parity(g, oracle.evaluate(b), ctx="sparse")
     assert g["stats"]["n_problems"] == _distinct_problems(b)
+
+
+def test_validation_fast_path_boundaries(sel):
+    """k_problem_w's validation shortcuts at their thresholds: access magnitudes
+    and extents just below / at 2^20 (below: no saturating bound arithmetic),
+    the address bound on either side of 2^62 (V6), per-access M_k below / above
+    2^26 (the 32-bit segmented sum of M_it) and P * M_it at 2^48 (V6; the valid
+    side of that boundary has ~2^43 warp-accesses, beyond the oracle)."""
+    import test_oracle_model as M
+    base = M.BASE
+    k20 = 1 << 20
+    acc = gen.make_access
+    items = [
+        dict(P0=100, trip=[], accesses=[acc(base=k20 - 4, c_par=(4,), elem_bytes=4)]),
+        dict(P0=100, trip=[], accesses=[acc(base=k20, c_par=(4,), elem_bytes=4)]),
+        dict(P0=k20 - 1, trip=[], accesses=[acc(base=base, c_par=(4,), elem_bytes=4)]),
+        dict(P0=k20, trip=[], accesses=[acc(base=base, c_par=(4,), elem_bytes=4)]),
+        dict(P0=64, trip=[k20 - 1], accesses=[acc(base=base, c_par=(4,), c_inner=(k20 - 4,), elem_bytes=4, depth=1)]),
+        dict(P0=64, trip=[3], accesses=[acc(base=base, c_par=(4,), c_inner=(k20,), elem_bytes=4, depth=1)]),
+        # |base| + |c| (P - 1) just below / at 2^62
+        dict(P0=2, trip=[], accesses=[acc(base=(1 << 62) - 8 - 4, c_par=(4,), elem_bytes=4)]),
+        dict(P0=2, trip=[], accesses=[acc(base=(1 << 62) - 4, c_par=(4,), elem_bytes=4)]),
+        # M_k = 2^13 * 2^13 = 2^26 on one access of a multi-access nest (64-bit segmented sum)
+        dict(P0=32, trip=[1 << 13, 1 << 13], accesses=[acc(base=base, c_par=(4,), elem_bytes=4),
+                                                      acc(base=base, c_par=(4,), c_inner=(4, 8), elem_bytes=4,
+                                                          depth=2)]),
+        # P M_it around 2^48 (ERANGE at and above)
+        dict(P0=1 << 20, trip=[1 << 14, 1 << 14], accesses=[acc(base=base, c_par=(4,), c_inner=(4, 8),
+                                                                elem_bytes=4, depth=2)]),
+    ]
+    b = gen.custom_batch(items)
+    ref = oracle.evaluate(b)
+    assert ref["status"][7] == 2 and ref["status"][6] == 0 and ref["status"][9] == 2
+    for flags in (0, 1):
+        g = run_gpu(sel, b, flags)
+        assert_parity(g, ref, ctx=f"validation boundaries flags={flags}")

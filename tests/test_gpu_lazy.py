@@ -59,7 +59,7 @@ def check(sel, b):
     for want_t in (True, False):
         ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), len(b))
         cands = sel._as_bytes_tensor(b.cands, "candidate")
-        r = ev.evaluate(cands, want_counts=True, want_t_gpu=want_t)
+        r = ev.evaluate(cands, want_counts=want_t, want_t_gpu=want_t)   # neither: the bench's loop instance
         torch.cuda.synchronize()
         g = {k: v.cpu().numpy() for k, v in r.items()}
         assert (g["status"] == ref["status"]).all()
@@ -134,3 +134,47 @@ def test_zero_cpu_cost_and_rep(sel):
     items = [dict(P0=p, trip=[], depth=0, comp=[9.0], accesses=[a], launch=li, device=gen.V100)
              for p in (32, 80 * 32, 81 * 32, 300 * 128, 10 ** 6 + 7) for li in (0, 1)]
     check(sel, gen.custom_batch(items, launches_=launches))
+
+
+def _plain(sel, b):
+    """decision / cycles / status only (the loop instance the bench times)."""
+    ev = sel.Evaluator((b.nests, b.accesses, b.launches, b.devices), max(len(b), 1))
+    r = ev.evaluate(sel._as_bytes_tensor(b.cands, "candidate"))
+    torch.cuda.synchronize()
+    return {k: v.cpu().numpy() for k, v in r.items()}
+
+
+@pytest.mark.parametrize("order", ["sweep", "shuffled", "reversed"])
+def test_plain_loop_any_order(sel, order):
+    """The candidate loop for direct ids with no t_gpu / counts stored (the
+    bench's instance) on c5's sweep order, a random permutation and the
+    reverse, with a batch that is not a multiple of any tile: the oracle's
+    bits."""
+    idx = np.arange(0, 5 * 768 + 77)
+    b = gen.generate_indices(5, 1000 * 768 + idx)
+    if order == "shuffled":
+        b = b.select(np.random.default_rng(3).permutation(len(b)))
+    elif order == "reversed":
+        b = b.select(np.arange(len(b))[::-1])
+    ref = oracle.evaluate(b)
+    g = _plain(sel, b)
+    assert (g["status"] == ref["status"]).all()
+    assert (g["decision"] == ref["decision"]).all()
+    assert (g["cycles"] == ref["cycles"]).all()
+
+
+def test_plain_loop_edges_and_device_counts(sel):
+    """Invalid and off-fast-path candidates in the bench's loop instance
+    (deferred to the exact path), with 4 and 3 device sets."""
+    b = gen.generate(2)
+    c = b.cands.copy()
+    c["cpu_hz"][5] = 0.0                          # V1 inside a run
+    c["launch_id"][9] = 200                       # V1: launch id out of range
+    c["cpu_cycles"][11] = 0.0                     # T_cpu = +0
+    b2 = gen.Batch(c, b.nests, b.accesses, b.launches, b.devices)
+    for bb in (b2, gen.Batch(c[c["device_id"] < 3], b.nests, b.accesses, b.launches, b.devices[:3])):
+        ref = oracle.evaluate(bb)
+        g = _plain(sel, bb)
+        assert (g["status"] == ref["status"]).all()
+        assert (g["decision"] == ref["decision"]).all()
+        assert (g["cycles"] == ref["cycles"]).all()

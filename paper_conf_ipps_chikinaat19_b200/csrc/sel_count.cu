@@ -1677,12 +1677,11 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
                         LANE_OPS(sOps += z[c].ops);
                         {   // the only writer so far (k_problem_w leaves these counters unzeroed): store
                             unsigned long long* pc = a.prob_cnt + q * kCntStride;
-                            if (a.hdr->n_parts == 1) {
-                                pc[0] = z[c].W;
-                                pc[1] = z[c].L;
-                                pc[2] = z[c].S;
-                                pc[3] = z[c].C;
-                                pc[4] = z[c].U;
+                            if (a.hdr->n_parts == 1) {         // the whole 48-byte record, M_it included
+                                ulonglong2* p2 = reinterpret_cast<ulonglong2*>(pc);
+                                p2[0] = make_ulonglong2(z[c].W, z[c].L);
+                                p2[1] = make_ulonglong2(z[c].S, z[c].C);
+                                p2[2] = make_ulonglong2(z[c].U, Mit);
                             } else if (z[c].W) {
                                 atomicAdd(pc + 0, (unsigned long long)z[c].W);
                                 atomicAdd(pc + 1, (unsigned long long)z[c].L);

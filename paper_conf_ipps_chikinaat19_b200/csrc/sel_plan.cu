@@ -302,7 +302,8 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
                                               const uint32_t* prob_B, unsigned long long* prob_W,
                                               unsigned long long* prob_WR, uint8_t* prob_status,
-                                              unsigned long long* prob_cnt, int lane_ok, bool one_part) {
+                                              unsigned long long* prob_cnt, int lane_ok, bool one_part,
+                                              bool lane_mit = false) {
     prob_status[q] = st;
     if (st) {
         for (int f = 0; f < kCntStride; f++) prob_cnt[q * kCntStride + f] = 0;
@@ -312,11 +313,13 @@ __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& ne
     }
     const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
     prob_WR[q] = WR;
-    prob_cnt[q * kCntStride + 5] = M_it;
     // small problems are counted one per lane (k_lane_problems), outside the prefix
     const uint64_t W = WR * M_it;
     const bool small = lane_ok && nest.par_dims == 1 && W <= kSmallMaxW && WR <= kSmallMaxWR;
     prob_W[q] = small ? 0ull : W;
+    // lane_mit: the lane kernel writes this problem's whole counter record,
+    // M_it included (one full 48-byte record instead of an 8-byte store here)
+    if (!(lane_mit && small && W != 0 && one_part)) prob_cnt[q * kCntStride + 5] = M_it;
     if (!(small && W != 0 && one_part))
         for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
     return (!small && W != 0 ? 1u : 0u) | (small && W != 0 ? 2u : 0u);
@@ -459,7 +462,7 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                     prob_B_w[q] = cls[kClsMax + c];
                     prob_used[q] = 0;
                     const uint32_t r = problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, prob_B, prob_W, prob_WR,
-                                                     prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
+                                                     prob_status, prob_cnt, lane_ok, hdr->n_parts == 1, c < 32);
                     big += r & 1u;
                     if (c < 32) lane_mask |= ((r >> 1) & 1u) << c;
                 }

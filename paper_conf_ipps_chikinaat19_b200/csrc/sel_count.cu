@@ -80,6 +80,20 @@ struct CountArgs {
     const uint32_t* cls_B;              // direct mode: B class of each class index
 };
 
+// nest and block size of problem q: derived from the id in direct mode
+// (q = nest * n_cls + class; k_problem_w does not materialise them there),
+// the plan's tables otherwise
+__device__ __forceinline__ void problem_nest_B(const CountArgs& a, uint64_t q, uint32_t& nid, uint32_t& B) {
+    if (a.hdr->direct) {
+        const uint32_t nc = a.hdr->n_cls;
+        nid = uint32_t(q / nc);
+        B = a.cls_B[q - uint64_t(nid) * nc];
+    } else {
+        nid = a.prob_nest[q];
+        B = a.prob_B[q];
+    }
+}
+
 // Accumulators of one warp for the problem being counted (<= kMaxChunk WAs).
 //   L = W + sum_lanes(lf) + lk      S = W + sum_lanes(sf) + sk
 //   C = C                           U = (W - C) + sum_lanes(uf) + uk
@@ -1174,9 +1188,10 @@ __device__ __noinline__ Acc expand_access(const sel_nest* np, const sel_access* 
 template <int MODE>
 __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint64_t off, uint32_t take, int lane,
                                            uint32_t* hist, WarpStats& st) {
-    const sel_nest* np = a.nests + a.prob_nest[q];
+    uint32_t nid, B;
+    problem_nest_B(a, q, nid, B);
+    const sel_nest* np = a.nests + nid;
     const sel_nest nest = *np;
-    const uint32_t B = a.prob_B[q];
     const uint64_t WR = a.prob_WR[q];
     const uint64_t P = nest.P0 * nest.P1;
     const uint64_t T0 = eff_trip(nest.trip[0]), T1 = eff_trip(nest.trip[1]), T2 = eff_trip(nest.trip[2]);
@@ -1774,8 +1789,9 @@ __global__ void __launch_bounds__(SEL_COUNT_THREADS, SEL_COUNT_MIN_BLOCKS) k_que
             const unsigned long long v = a.queue[e0 + lane];
             q_l = uint32_t(v >> 32);
             hm_l = uint32_t(v);
-            const sel_nest* np = a.nests + a.prob_nest[q_l];
-            B_l = a.prob_B[q_l];
+            uint32_t nid_l;
+            problem_nest_B(a, q_l, nid_l, B_l);
+            const sel_nest* np = a.nests + nid_l;
             WR_l = uint32_t(a.prob_WR[q_l]);
             P_l = uint32_t(np->P0);
             T0_l = uint32_t(eff_trip(np->trip[0]));

@@ -300,7 +300,7 @@ __global__ void k_finalize_plan(WsHeader* hdr, const unsigned long long* nest_ba
 // (k_queue adds the handed-over accesses afterwards).
 // returns bit 0: counted through the WA prefix (big), bit 1: counted by the lane kernel (small, W > 0)
 __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& nest, uint8_t st, uint64_t M_it,
-                                              const uint32_t* prob_B, unsigned long long* prob_W,
+                                              uint32_t B, unsigned long long* prob_W,
                                               unsigned long long* prob_WR, uint8_t* prob_status,
                                               unsigned long long* prob_cnt, int lane_ok, bool one_part,
                                               bool lane_mit = false) {
@@ -311,7 +311,7 @@ __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& ne
         prob_WR[q] = 0;
         return 0u;
     }
-    const uint64_t WR = warp_reps(nest.P0 * nest.P1, prob_B[q]);
+    const uint64_t WR = warp_reps(nest.P0 * nest.P1, B);
     prob_WR[q] = WR;
     // small problems are counted one per lane (k_lane_problems), outside the prefix
     const uint64_t W = WR * M_it;
@@ -333,6 +333,8 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                                                    uint8_t* prob_used, uint2* lane_info) {
     const uint64_t nq = hdr->n_problems;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    (void)prob_nest_w;                                      // direct mode no longer materialises nest / B per
+    (void)prob_B_w;                                         // problem (problem_nest_B derives them)
     if (hdr->direct) {
         // direct ids: the problems of nest i are i * n_cls + [0, n_cls), every
         // one of them counted (direct mode requires n_nests * n_cls <= n, so
@@ -458,11 +460,11 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
                 for (uint32_t c = 0; c < ncls; c++) {
                     const uint64_t q = i * ncls + c;
                     used++;
-                    prob_nest_w[q] = uint32_t(i);
-                    prob_B_w[q] = cls[kClsMax + c];
-                    prob_used[q] = 0;
-                    const uint32_t r = problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, prob_B, prob_W, prob_WR,
-                                                     prob_status, prob_cnt, lane_ok, hdr->n_parts == 1, c < 32);
+                    // (nest and B of a direct id are derived where needed: problem_nest_B)
+                    const uint32_t r = problem_w_one(q, nest, st, st == SEL_OK ? M_it : 0ull, cls[kClsMax + c],
+                                                     prob_W, prob_WR, prob_status, prob_cnt, lane_ok,
+                                                     hdr->n_parts == 1, c < 32);
+                    if (r & 1u) prob_used[q] = 0;              // k_mark_big / k_drop_unused look at big ones only
                     big += r & 1u;
                     if (c < 32) lane_mask |= ((r >> 1) & 1u) << c;
                 }
@@ -488,7 +490,8 @@ __global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, 
             nest = t.nests[nid];
             st = validate_nest(nest, t.accesses, t.n_accesses, &M_it);
         }
-        problem_w_one(q, nest, st, M_it, prob_B, prob_W, prob_WR, prob_status, prob_cnt, lane_ok, hdr->n_parts == 1);
+        problem_w_one(q, nest, st, M_it, prob_B[q], prob_W, prob_WR, prob_status, prob_cnt, lane_ok,
+                      hdr->n_parts == 1);
     }
 }
 

@@ -15,7 +15,10 @@ constexpr uint64_t kLim40 = 1ull << 40;
 constexpr uint32_t kNoProblem = 0xffffffffu;
 constexpr int kSlots = 8;              // distinct B classes shared per nest before overflow
 constexpr uint32_t kClsMax = 1024;     // launch tables up to this size use direct problem ids
-constexpr int kCntStride = 6;          // per problem: W, L, S, C, U (atomic), M_it (closed form)
+#ifndef SEL_CNT_STRIDE
+#define SEL_CNT_STRIDE 6
+#endif
+constexpr int kCntStride = SEL_CNT_STRIDE;   // per problem: W, L, S, C, U (atomic), M_it (closed form)[, pad]
 constexpr size_t kProbModelBytes = 112; // per problem: the candidate-independent part of a4 (sel_model.cu)
 
 // ------------------------------------------------------------------ workspace

@@ -321,7 +321,7 @@ __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& ne
     // M_it included (one full 48-byte record instead of an 8-byte store here)
     if (!(lane_mit && small && W != 0 && one_part)) prob_cnt[q * kCntStride + 5] = M_it;
     if (!(small && W != 0 && one_part))
-        for (int f = 0; f < kCntStride - 1; f++) prob_cnt[q * kCntStride + f] = 0;
+        for (int f = 0; f < 5; f++) prob_cnt[q * kCntStride + f] = 0;     // W, L, S, C, U
     return (!small && W != 0 ? 1u : 0u) | (small && W != 0 ? 2u : 0u);
 }
 

@@ -1516,8 +1516,21 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
     // (c5: 3.1 M nests), else the units spread over the grid in tiles of at
     // least 512 (small batches no longer run on a few blocks)
     const uint64_t per_block = (ue - ub + gridDim.x - 1) / gridDim.x;
+#ifndef SEL_LANE_BALANCE
+#define SEL_LANE_BALANCE 1
+#endif
+#if SEL_LANE_BALANCE
+    // the fewest waves of tiles of <= kLaneTile units, and the tile size that
+    // fills the last wave (c5: 3.1 M nests on 296 blocks -> 3 waves of 3584,
+    // not 2.58 waves of 4096 whose last wave leaves 42 % of the blocks idle)
+    const uint64_t waves = (per_block + kLaneTile - 1) / kLaneTile;
+    const uint64_t per_wave = waves ? (per_block + waves - 1) / waves : 0;
+    const uint32_t tile = uint32_t(per_wave <= 512 ? 512u
+                                   : umin64(((per_wave + kLaneThreads - 1) / kLaneThreads) * kLaneThreads, kLaneTile));
+#else
     const uint32_t tile = uint32_t(per_block >= kLaneTile ? kLaneTile
                                    : per_block <= 512 ? 512u : ((per_block + kLaneThreads - 1) / kLaneThreads) * kLaneThreads);
+#endif
     for (uint64_t t0 = ub + uint64_t(blockIdx.x) * tile; t0 < ue; t0 += uint64_t(gridDim.x) * tile) {
         const uint32_t nt = uint32_t(umin64(tile, ue - t0));
         // ---- sort the tile's units by shape key (counting sort in shared memory)

@@ -325,7 +325,10 @@ __device__ __forceinline__ uint32_t problem_w_one(uint64_t q, const sel_nest& ne
     return (!small && W != 0 ? 1u : 0u) | (small && W != 0 ? 2u : 0u);
 }
 
-__global__ void __launch_bounds__(256) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
+#ifndef SEL_PW_MIN_BLOCKS
+#define SEL_PW_MIN_BLOCKS 4      // 64 registers, 4 blocks per SM: 0.386 -> 0.349 ms (3 blocks at 78 registers before)
+#endif
+__global__ void __launch_bounds__(256, SEL_PW_MIN_BLOCKS) k_problem_w(sel_tables t, WsHeader* hdr, const uint32_t* prob_nest,
                                                    const uint32_t* prob_B, unsigned long long* prob_W,
                                                    unsigned long long* prob_WR, uint8_t* prob_status,
                                                    unsigned long long* prob_cnt, int lane_ok, uint8_t* nest_key,

@@ -320,8 +320,11 @@ def run_ours(args):
             gatherer.wait()
 
     int_peak = {"alu": sel.int_peak(0), "fma": sel.int_peak(1), "both": sel.int_peak(2)}
+    nvtx = torch.cuda.nvtx                      # host-timeline ranges (the library adds sel:plan/count/model)
+    nvtx.range_push("bench:warmup")
     for _ in range(args.warmup):
         step()
+    nvtx.range_pop()
     torch.cuda.synchronize(dev)
     stats = {}
     for sh in shards:
@@ -340,8 +343,10 @@ def run_ours(args):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         e0.record(stream)
-        for _ in range(args.steps):
+        for k in range(args.steps):
+            nvtx.range_push(f"bench:step {k}")
             step()
+            nvtx.range_pop()
         e1.record(stream)
         torch.cuda.synchronize(dev)
     D.barrier(world)
@@ -389,8 +394,10 @@ def run_ours(args):
         else:
             f0.record(join)
         for k in range(args.steps):
+            nvtx.range_push(f"bench:e2e step {k}")
             for p, ch, nh, ah in pipes:
                 p.step(k, ch, nh, ah)
+            nvtx.range_pop()
         for p, _, _, _ in pipes:
             join.wait_stream(p.d2h)
         f1.record(join)

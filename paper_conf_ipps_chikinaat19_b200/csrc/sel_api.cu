@@ -7,6 +7,7 @@
 #include <cstring>
 #include <mutex>
 #include <vector>
+#include <nvtx3/nvToolsExt.h>
 #include "sel_device.cuh"
 #include "sel_internal.h"
 
@@ -46,14 +47,27 @@ static cudaEvent_t prof_event() {
     return e;
 }
 
+// NVTX ranges (tracing) around the same regions, on the host
+// timeline of the enqueueing thread: a no-op unless a tool is attached.
+static const char* const kProfNames[SEL_PROF_REGIONS] = {"sel:plan", "sel:count", "sel:model",
+                                                         "sel:k_model_fused", "sel:k_lane_problems",
+                                                         "sel:k_problem_w"};
+static nvtxRangeId_t g_nvtx[SEL_PROF_REGIONS] = {};
+
 void prof_begin(int region, cudaStream_t s) {
     std::lock_guard<std::mutex> g(g_prof_mu);
+    if (g_nvtx[region]) nvtxRangeEnd(g_nvtx[region]);
+    g_nvtx[region] = nvtxRangeStartA(kProfNames[region]);
     if (!g_prof_on) return;
     g_prof_cur_begin[region] = prof_event();
     cudaEventRecord(g_prof_cur_begin[region], s);
 }
 void prof_end(int region, cudaStream_t s) {
     std::lock_guard<std::mutex> g(g_prof_mu);
+    if (g_nvtx[region]) {
+        nvtxRangeEnd(g_nvtx[region]);
+        g_nvtx[region] = 0;
+    }
     if (!g_prof_on || !g_prof_cur_begin[region]) return;
     cudaEvent_t e = prof_event();
     cudaEventRecord(e, s);

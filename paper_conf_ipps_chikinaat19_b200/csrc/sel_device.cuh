@@ -169,19 +169,25 @@ __device__ __forceinline__ uint32_t access_check(const sel_access& a, uint32_t p
     if (bad) return kAccInval;
     const uint64_t e0 = (par_dims == 1) ? P : P0;
     {
-        // every magnitude and extent below 2^20: each of the <= 6 bound terms is
-        // below 2^40, so the bound is far below 2^62 and M_k (<= 3 trips) below
-        // 2^60 -- no saturating arithmetic needed (the common case)
-        uint64_t big = uabs(a.base) | uabs(a.c_par[0]) | e0;
-        if (par_dims == 2) big |= uabs(a.c_par[1]) | P1;
+        // |base| < 2^60, every coefficient below 2^28 and every extent below
+        // 2^20: each of the <= 5 product terms is below 2^48, so the bound stays
+        // below 2^61 < 2^62 and M_k (<= 3 trips) below 2^60 -- no saturating
+        // arithmetic needed (the common case: array bases are large, strides
+        // and trip counts small)
+        uint64_t coef = uabs(a.c_par[0]), ext = e0;
+        if (par_dims == 2) {
+            coef |= uabs(a.c_par[1]);
+            ext |= P1;
+        }
         uint64_t Mk = 1;
 #pragma unroll
         for (int j = 0; j < 3; j++)
             if (j < a.depth) {
-                big |= uabs(a.c_inner[j]) | T[j];
+                coef |= uabs(a.c_inner[j]);
+                ext |= T[j];
                 Mk *= T[j];
             }
-        if ((big >> 20) == 0) {
+        if (((uabs(a.base) >> 60) | (coef >> 28) | (ext >> 20)) == 0) {
             *Mk_out = Mk;
             return 0u;
         }

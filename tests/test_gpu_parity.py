@@ -611,8 +611,9 @@ def test_direct_ids_sparse_nests(sel):
 
 
 def test_validation_fast_path_boundaries(sel):
-    """k_problem_w's validation shortcuts at their thresholds: access magnitudes
-    and extents just below / at 2^20 (below: no saturating bound arithmetic),
+    """k_problem_w's validation shortcuts at their thresholds: |base| 2^60,
+    coefficients 2^28, extents 2^20 (below all three: no saturating bound
+    arithmetic),
     the address bound on either side of 2^62 (V6), per-access M_k below / above
     2^26 (the 32-bit segmented sum of M_it) and P * M_it at 2^48 (V6; the valid
     side of that boundary has ~2^43 warp-accesses, beyond the oracle)."""
@@ -627,6 +628,13 @@ def test_validation_fast_path_boundaries(sel):
         dict(P0=k20, trip=[], accesses=[acc(base=base, c_par=(4,), elem_bytes=4)]),
         dict(P0=64, trip=[k20 - 1], accesses=[acc(base=base, c_par=(4,), c_inner=(k20 - 4,), elem_bytes=4, depth=1)]),
         dict(P0=64, trip=[3], accesses=[acc(base=base, c_par=(4,), c_inner=(k20,), elem_bytes=4, depth=1)]),
+        # the shortcut's own thresholds: |base| 2^60, coefficients 2^28
+        dict(P0=100, trip=[], accesses=[acc(base=(1 << 60) - 4, c_par=(4,), elem_bytes=4)]),
+        dict(P0=100, trip=[], accesses=[acc(base=1 << 60, c_par=(4,), elem_bytes=4)]),
+        dict(P0=100, trip=[3], accesses=[acc(base=base, c_par=((1 << 28) - 4,), c_inner=((1 << 28) - 8,),
+                                             elem_bytes=4, depth=1)]),
+        dict(P0=100, trip=[3], accesses=[acc(base=base, c_par=(1 << 28,), c_inner=(1 << 28,), elem_bytes=4,
+                                             depth=1)]),
         # |base| + |c| (P - 1) just below / at 2^62
         dict(P0=2, trip=[], accesses=[acc(base=(1 << 62) - 8 - 4, c_par=(4,), elem_bytes=4)]),
         dict(P0=2, trip=[], accesses=[acc(base=(1 << 62) - 4, c_par=(4,), elem_bytes=4)]),
@@ -640,7 +648,7 @@ def test_validation_fast_path_boundaries(sel):
     ]
     b = gen.custom_batch(items)
     ref = oracle.evaluate(b)
-    assert ref["status"][7] == 2 and ref["status"][6] == 0 and ref["status"][9] == 2
+    assert ref["status"][11] == 2 and ref["status"][10] == 0 and ref["status"][13] == 2
     for flags in (0, 1):
         g = run_gpu(sel, b, flags)
         assert_parity(g, ref, ctx=f"validation boundaries flags={flags}")

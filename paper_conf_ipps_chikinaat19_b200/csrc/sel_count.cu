@@ -1256,6 +1256,9 @@ __device__ __noinline__ void count_problem(const CountArgs& a, uint64_t q, uint6
 // the lane); at the first access that needs the warp (deeper loop nests, block
 // sizes whose warp-reps fall into many residue classes, collapse(2)) it hands
 // the rest of its problem to the warp (queue of <= 32 entries).
+#ifndef SEL_LANE_DYN
+#define SEL_LANE_DYN 1      // warps take 32-nest chunks of a tile dynamically
+#endif
 #ifndef SEL_LANE_PF
 #define SEL_LANE_PF 1       // L1 prefetch of the nest's next access descriptors (2: + the next nest into L2)
 #endif
@@ -1501,6 +1504,9 @@ __device__ __forceinline__ uint32_t lane_unit_key(const CountArgs& a, uint64_t u
 template <int MODE>
 __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_problems(const __grid_constant__ CountArgs a) {
     extern __shared__ uint32_t s_lane[];                    // hist columns | tile order | key counts
+#if SEL_LANE_DYN
+    __shared__ uint32_t s_next;                             // next 32-nest chunk of the tile
+#endif
     uint32_t* s_order = s_lane + kLaneRows * kLaneThreads;
     uint32_t* s_cnt = s_order + kLaneTile;
     const Col hcol{s_lane + threadIdx.x};
@@ -1535,6 +1541,9 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
         const uint32_t nt = uint32_t(umin64(tile, ue - t0));
         // ---- sort the tile's units by shape key (counting sort in shared memory)
         for (uint32_t i = threadIdx.x; i < kLaneKeys; i += blockDim.x) s_cnt[i] = 0u;
+#if SEL_LANE_DYN
+        if (threadIdx.x == 0) s_next = 0u;
+#endif
         __syncthreads();
         uint32_t key[kLaneTile / kLaneThreads];
 #pragma unroll
@@ -1566,8 +1575,20 @@ __global__ void __launch_bounds__(kLaneThreads, SEL_LANE_MIN_BLOCKS) k_lane_prob
         }
         __syncthreads();
         // ---- count: round r, thread t takes the unit at sorted position r * threads + t
+#if SEL_LANE_DYN
+        // warps take 32-nest chunks of the sorted tile from a shared counter:
+        // chunks of different shapes cost different times, and a static round
+        // assignment left warps idle at the end-of-tile barrier
+        for (;;) {
+            uint32_t chunk = 0;
+            if (lane == 0) chunk = atomicAdd(&s_next, 1u);
+            chunk = __shfl_sync(kFull, chunk, 0);
+            if (chunk * 32u >= nt) break;
+            const uint32_t i = chunk * 32u + uint32_t(lane);
+#else
         for (uint32_t r = 0; r * kLaneThreads < nt; r++) {
             const uint32_t i = r * kLaneThreads + threadIdx.x;
+#endif
             const bool has = i < nt;
             const uint64_t u = has ? t0 + s_order[i] : 0ull;
 #if SEL_LANE_PF >= 2
